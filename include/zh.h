@@ -1,0 +1,190 @@
+/* zh.h — C ABI of libzh, the B200-native (sm_100a) zonal-histogramming library.
+ *
+ * Operation (§III ¶1): given a raster R (M rows x N columns, integer values) and
+ * polygons P_k, compute for every polygon the histogram
+ *     H_k[b] = #{ cells (i, j) : centre of (i, j) inside P_k  and  bin(R[i][j]) = b }.
+ * The cell CENTRE is the representative point (§III.D); "inside" is the even-odd
+ * ray-crossing test of Franklin's PNPOLY over all rings of the polygon (Fig. 5 and
+ * the multi-ring paragraph after it), evaluated in IEEE double with canonical edge orientation
+ * and no FMA contraction (readings R7/R8/R10).
+ *
+ * The paper's four steps (§I, §III ¶1 and Fig. 1) are exposed one call
+ * per step so each can be timed and tested:
+ *   step 1 zh_tile_hist   per-tile histograms of T x T tiles           (PAPER.md:14 §III.A, :16 Fig. 2)
+ *   step 2 zh_pair_tiles  MBB rasterisation pairing + inside/outside/intersect classification
+ *                                                                        (§III.B, Fig. 3)
+ *   step 3 zh_aggregate   add inside tiles' histograms to the polygons  (§III.C, Fig. 4)
+ *   step 4 zh_pip_update  cell-in-polygon test for the cells of intersecting tiles
+ *                                                                        (§III.D, Fig. 5)
+ *   zh_run                steps 2, 1, 3, 4 and the copy of the result to the host.
+ *
+ * Conventions
+ *  - Every call returns zh_status; nothing throws, exits or prints.  On failure
+ *    zh_last_error() returns a thread-local message.  A failed call leaves the context usable;
+ *    after ZH_ERR_CUDA the device state (and the output) is unspecified.
+ *  - All device work is enqueued on options.stream (a cudaStream_t, NULL = legacy default
+ *    stream).  Calls documented "syncs" block the host until the stream has drained.
+ *  - Ownership: the raster is BORROWED (caller keeps it alive for the context's lifetime);
+ *    polygons and bin parameters are COPIED by zh_create; tile histograms, pair lists and the
+ *    output are OWNED by the context unless zh_set_output supplied a borrowed output buffer.
+ *  - Index widths: offsets are int64 at the ABI; kernels use int32 internally, so n_vert,
+ *    n_ring, the number of tiles and the number of tile/polygon pairs must stay < 2^31
+ *    (else ZH_ERR_UNSUPPORTED).
+ *  - Threading: a context is used by one host thread at a time.
+ */
+#ifndef ZH_H
+#define ZH_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ZH_ABI_VERSION 1
+
+typedef struct zh_ctx_s* zh_ctx;
+
+typedef enum {
+  ZH_OK = 0,
+  ZH_ERR_INVALID_ARG = 1,  /* malformed input (see zh_create)                                 */
+  ZH_ERR_UNSUPPORTED = 2,  /* valid but outside what the kernels support (rotated gt, >2^31)  */
+  ZH_ERR_OOM = 3,          /* device allocation failed                                        */
+  ZH_ERR_CUDA = 4,         /* a CUDA runtime error; message has the CUDA error string         */
+  ZH_ERR_OVERFLOW = 5,     /* out_u64 = 0 requested but a count could exceed 2^32 - 1         */
+  ZH_ERR_STATE = 6         /* call order violated (e.g. zh_aggregate before steps 1 and 2)     */
+} zh_status;
+
+/* Raster shard.  `data` points at the first element of row `row0` of the full raster.
+ * Layout: row-major int16, `pitch` elements between consecutive rows (pitch >= cols).
+ * on_host = 0: `data` is DEVICE memory (borrowed).  The fast paths need data % 16 == 0 and
+ *   pitch % 8 == 0 (16-byte vector loads); other alignments are rejected (INVALID_ARG).
+ * on_host = 1: `data` is HOST memory (borrowed; pin it for full PCIe speed); the context owns a
+ *   device copy and every zh_run / zh_upload_raster copies the shard host->device first.
+ * Geotransform (GDAL): x = gt[0] + col*gt[1] + row*gt[2], y = gt[3] + col*gt[4] + row*gt[5];
+ *   the cell (r, c) has centre x = gt[0] + (c + 0.5)*gt[1], y = gt[3] + (r + 0.5)*gt[5].
+ *   gt[2] and gt[4] must be 0 (north-up; rotated -> UNSUPPORTED); gt[1], gt[5] nonzero, finite.
+ * Sharding (multi-GPU): a rank holds rows [row0, row0 + nrows) of an M x N raster; row0 must be
+ *   a multiple of the tile size so that shards consist of whole tile rows. */
+typedef struct {
+  const int16_t* data;
+  int64_t rows, cols;     /* full raster M, N                                                   */
+  int64_t pitch;          /* elements between rows of `data`                                    */
+  int64_t row0, nrows;    /* this shard's rows                                                  */
+  double gt[6];
+  int32_t on_host;
+  int32_t reserved;
+} zh_raster;
+
+/* Polygons, HOST arrays, copied by zh_create (the caller may free them afterwards).
+ * Polygon k owns rings poly_ring_off[k] .. poly_ring_off[k+1]-1; ring r owns vertices
+ * ring_vert_off[r] .. ring_vert_off[r+1]-1.  Rings are closed implicitly (edge from the last
+ * vertex back to the first); an explicit closing vertex is allowed and adds a zero-length edge.
+ * Holes and multi-part polygons are just more rings (even-odd rule over all rings of a polygon,
+ * the semantics of the paper's origin-sentinel trick).  Degenerate input is valid:
+ * polygons with no rings, rings with 0-2 vertices, zero-area rings, polygons off the raster all
+ * contribute nothing.  Offsets must be non-decreasing with [0] = 0 and the last = n_ring /
+ * n_vert; coordinates finite (else INVALID_ARG). */
+typedef struct {
+  int64_t n_poly, n_ring, n_vert;
+  const int64_t* poly_ring_off; /* n_poly + 1 */
+  const int64_t* ring_vert_off; /* n_ring + 1 */
+  const double* x;              /* n_vert     */
+  const double* y;              /* n_vert     */
+} zh_polygons;
+
+/* Bin mapping (DESIGN.md §3 R3/R4; the paper assumes 0 <= v < B, and Fig. 2 does
+ * no check):  a cell with use_nodata && v == nodata is never counted; otherwise
+ * d = v - lo; d < 0 -> bin 0 (clamp) or not counted (oor_drop); b = d / width;
+ * b >= nbins -> nbins-1 (clamp) or not counted (oor_drop).
+ * Requires 1 <= nbins <= 1<<20, 1 <= width, |lo| <= 1<<30. */
+typedef struct {
+  int32_t lo, width, nbins;
+  int32_t use_nodata, nodata;
+  int32_t oor_drop;
+} zh_bins;
+
+typedef struct {
+  int32_t tile;        /* T >= 1, arbitrary ("allow users to set it arbitrarily");
+                          partial edge tiles hold only real cells                                */
+  int32_t out_u64;     /* 1: uint64 output (default); 0: uint32 (ZH_ERR_OVERFLOW at zh_create if
+                          some polygon's MBB could hold >= 2^32 cells)                           */
+  int32_t force_isect; /* 1: classify every non-outside pair as intersecting (skips step 3's
+                          work; a validation mode — the result must not change)                  */
+  int32_t reserved;
+  void* stream;        /* cudaStream_t                                                          */
+} zh_options;
+
+typedef struct {
+  int64_t n_tiles;        /* tiles of this shard                                                */
+  int64_t n_candidates;   /* (tile, polygon) pairs from MBB rasterisation                      */
+  int64_t n_inside;       /* pairs classified inside (step 3 work)                              */
+  int64_t n_isect;        /* pairs classified intersecting (step 4 work)                        */
+  int64_t n_band_entries; /* (edge, tile-row) entries of the step-4 edge lists                  */
+  int64_t n_edges;        /* polygon edges                                                      */
+  int64_t device_bytes;   /* device memory owned by the context                                 */
+} zh_stats;
+
+/* Validate, copy polygons to the device (H2D on options->stream), allocate per-tile histograms
+ * and the output.  *out is set only on ZH_OK. */
+zh_status zh_create(zh_ctx* out, const zh_raster* raster, const zh_polygons* polys, const zh_bins* bins,
+                    const zh_options* options);
+
+/* on_host rasters: enqueue the host->device copy of the shard (zh_run does this itself). */
+zh_status zh_upload_raster(zh_ctx ctx);
+
+/* Step 1 (async): tile_hist[t][b] for every tile t of the shard. */
+zh_status zh_tile_hist(zh_ctx ctx);
+
+/* Step 2: edge preparation, MBB pairing, classification, pair lists; zeroes the output.
+ * Syncs the stream (twice) to size its lists.  n_inside / n_isect may be NULL. */
+zh_status zh_pair_tiles(zh_ctx ctx, int64_t* n_inside, int64_t* n_isect);
+
+/* Step 3 (async): out[k][b] += sum of tile_hist[t][b] over inside tiles t of k.
+ * Needs steps 1 and 2 since the last zh_pair_tiles, else ZH_ERR_STATE. */
+zh_status zh_aggregate(zh_ctx ctx);
+
+/* Step 4 (async): for every intersecting (tile, polygon) pair and every cell of the tile whose
+ * centre is inside the polygon, out[k][bin(v)] += 1.  Needs step 2, else ZH_ERR_STATE. */
+zh_status zh_pip_update(zh_ctx ctx);
+
+/* Upload (on_host), steps 2, 1, 3, 4, then copy n_poly * nbins elements (uint64 or uint32 per
+ * out_u64, row-major [n_poly][nbins]) to host_out (may be NULL to skip the copy).  Syncs. */
+zh_status zh_run(zh_ctx ctx, void* host_out);
+
+/* BORROWED device pointer to the output ([n_poly][nbins], uint64 or uint32) — e.g. for an
+ * NCCL reduce across shards.  *n = n_poly * nbins elements. */
+zh_status zh_output_device(zh_ctx ctx, void** dptr, int64_t* n);
+
+/* Use a caller-owned device buffer (n_poly * nbins elements, 8-byte aligned) as the output
+ * from now on (BORROWED, must outlive the context).  NULL reverts to the context's own. */
+zh_status zh_set_output(zh_ctx ctx, void* dptr);
+
+/* Copy the per-tile histograms of the shard ([n_tiles][nbins] uint32, tile id = local tile row *
+ * tile columns + tile column) to host memory (testing/inspection).  Syncs. */
+zh_status zh_copy_tile_hist(zh_ctx ctx, uint32_t* host, int64_t n_elems);
+
+/* Copy step 2's pair lists to host memory (testing).  inside: n_inside (tile, poly) int32 pairs;
+ * isect: n_isect (tile, poly) int32 pairs; either may be NULL.  Syncs. */
+zh_status zh_copy_pairs(zh_ctx ctx, int32_t* inside, int32_t* isect);
+
+zh_status zh_get_stats(zh_ctx ctx, zh_stats* stats);
+
+/* Per-step device time (ms) of the last call of each step, measured with CUDA events on the
+ * context stream when timing is enabled (zh_set_timing).  ms[0..3] = steps 1..4. */
+zh_status zh_set_timing(zh_ctx ctx, int32_t enable);
+zh_status zh_get_step_ms(zh_ctx ctx, float* ms4);
+
+/* Number of kernel launches the context has enqueued since creation (self-reported). */
+int64_t zh_launch_count(zh_ctx ctx);
+
+const char* zh_last_error(void);
+int32_t zh_abi_version(void);
+
+/* Frees the context's device memory (after synchronising its stream). NULL is a no-op. */
+void zh_destroy(zh_ctx ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ZH_H */

@@ -1,0 +1,444 @@
+// k_pairs.cu — step 2: pair raster tiles with polygons and classify each pair
+// (§III.B, Fig. 3; segment bookkeeping of PAPER.md:16-18 §III.C / Fig. 4 left).
+//
+// Paper design (prior art): MBB rasterisation with the GPU grid-file of [19]; the tile-in-polygon
+// test on the CPU "using well-established computational geometry libraries", then Thrust
+// stable_sort_by_key / stable_partition / reduce_by_key / scan to build per-polygon segments.
+// B200 design, all on the GPU:
+//   1. k_edges   — one thread per vertex: the ring edge it starts, in canonical orientation, and
+//                  the exact half-open interval of centre rows it straddles (ya <= yc(r) < yb),
+//                  found with the same yc(r) expression the PIP test uses;
+//   2. k_mbb     — one CTA per polygon: vertex MBB -> covered tile rectangle (1-cell margin);
+//   3. scans     — candidate offsets and band (polygon, tile-row) bases (CUB);
+//   4. k_band_*  — per (polygon, tile row) lists of the edges whose row interval meets it (the
+//                  step-4 edge lists and the classifier's input);
+//   5. k_mark    — a tile is INTERSECT if some edge's bounding box comes within one cell of
+//                  its cell rectangle (conservative; DESIGN.md §4 proof);
+//   6. k_classify— every other candidate tile has a uniform computed PIP status, evaluated exactly
+//                  at its first cell with a scanline over the band's edges (INSIDE / OUTSIDE);
+//   7. compaction— packed (inside, intersect) exclusive scan -> (tile, polygon) lists sorted by
+//                  (polygon, tile).
+#include <cub/device/device_scan.cuh>
+
+#include "zh_ctx.h"
+
+namespace zh {
+
+__device__ __forceinline__ int upper_bound_i32(const int32_t* a, int n, int32_t v) {
+  int lo = 0, hi = n;  // first index with a[i] > v
+  while (lo < hi) {
+    int m = (lo + hi) >> 1;
+    if (a[m] <= v) lo = m + 1; else hi = m;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int64_t upper_bound_i64(const int64_t* a, int64_t n, int64_t v) {
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    int64_t m = (lo + hi) >> 1;
+    if (a[m] <= v) lo = m + 1; else hi = m;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int64_t clamp_est(double v, int64_t lo, int64_t hi) {
+  if (!(v > (double)lo)) return lo;  // also NaN
+  if (v > (double)hi) return hi;
+  return (int64_t)ceil(v);
+}
+
+// Rows r in [rA, rB) with ya <= yc(r) < yb, exactly (monotone predicates + first_false).
+__device__ __forceinline__ int2 straddle_rows(const Geo& g, double ya, double yb, int64_t rA, int64_t rB) {
+  if (!(ya < yb)) return make_int2(0, 0);
+  const double ea = (ya - g.gt3) / g.gt5 - 0.5, eb = (yb - g.gt3) / g.gt5 - 0.5;
+  int64_t ra, rb;
+  if (g.gt5 < 0) {  // yc decreasing in r
+    // B(r): yc(r) < yb  is false then true -> ra = first r with B true
+    ra = first_false(rA, rB, clamp_est(eb, rA, rB), [&](int64_t r) { return !(row_centre(g, r) < yb); });
+    // A(r): ya <= yc(r) is true then false -> rb = first r with A false
+    rb = first_false(rA, rB, clamp_est(ea, rA, rB), [&](int64_t r) { return ya <= row_centre(g, r); });
+  } else {          // yc increasing in r
+    ra = first_false(rA, rB, clamp_est(ea, rA, rB), [&](int64_t r) { return !(ya <= row_centre(g, r)); });
+    rb = first_false(rA, rB, clamp_est(eb, rA, rB), [&](int64_t r) { return row_centre(g, r) < yb; });
+  }
+  if (ra >= rb) return make_int2(0, 0);
+  return make_int2((int)ra, (int)rb);
+}
+
+__global__ void k_edges(const int32_t* __restrict__ pro, int P, const int32_t* __restrict__ rvo, int R,
+                        const double* __restrict__ x, const double* __restrict__ y, int V, Geo g,
+                        int64_t rA, int64_t rB, int T, Edge* __restrict__ edges, int2* __restrict__ erows,
+                        int32_t* __restrict__ epoly, int32_t* __restrict__ espan) {
+  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    const int ring = upper_bound_i32(rvo, R + 1, v) - 1;
+    const int poly = upper_bound_i32(pro, P + 1, ring) - 1;
+    const int nxt = (v + 1 < rvo[ring + 1]) ? v + 1 : rvo[ring];
+    const double x0 = x[v], y0 = y[v], x1 = x[nxt], y1 = y[nxt];
+    Edge e;
+    if (y0 <= y1) { e.xa = x0; e.ya = y0; e.xb = x1; e.yb = y1; }
+    else          { e.xa = x1; e.ya = y1; e.xb = x0; e.yb = y0; }
+    edges[v] = e;
+    const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
+    erows[v] = rr;
+    epoly[v] = poly;
+    espan[v] = (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
+  }
+}
+
+// One CTA per polygon: MBB of its vertices -> covered tile rectangle (global tile indices),
+// clipped to the raster columns and the shard rows.  Empty -> (1, 0, 1, 0).
+__global__ void __launch_bounds__(256) k_mbb(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                              const double* __restrict__ x, const double* __restrict__ y, Geo g,
+                                              RasterP rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
+                                              int64_t* __restrict__ nband) {
+  const int k = blockIdx.x;
+  const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
+  double xmn = INFINITY, xmx = -INFINITY, ymn = INFINITY, ymx = -INFINITY;
+  for (int i = vb + threadIdx.x; i < ve; i += blockDim.x) {
+    xmn = fmin(xmn, x[i]); xmx = fmax(xmx, x[i]);
+    ymn = fmin(ymn, y[i]); ymx = fmax(ymx, y[i]);
+  }
+  __shared__ double s[4][8];
+  for (int o = 16; o > 0; o >>= 1) {
+    xmn = fmin(xmn, __shfl_xor_sync(0xffffffffu, xmn, o));
+    xmx = fmax(xmx, __shfl_xor_sync(0xffffffffu, xmx, o));
+    ymn = fmin(ymn, __shfl_xor_sync(0xffffffffu, ymn, o));
+    ymx = fmax(ymx, __shfl_xor_sync(0xffffffffu, ymx, o));
+  }
+  const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) { s[0][wid] = xmn; s[1][wid] = xmx; s[2][wid] = ymn; s[3][wid] = ymx; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int w = 1; w < (int)(blockDim.x >> 5); ++w) {
+      xmn = fmin(xmn, s[0][w]); xmx = fmax(xmx, s[1][w]);
+      ymn = fmin(ymn, s[2][w]); ymx = fmax(ymx, s[3][w]);
+    }
+    int4 m = make_int4(1, 0, 1, 0);
+    int64_t nc = 0, nb = 0;
+    if (ve > vb) {
+      double ca = (xmn - g.gt0) / g.gt1, cb = (xmx - g.gt0) / g.gt1;
+      double ra = (ymn - g.gt3) / g.gt5, rb = (ymx - g.gt3) / g.gt5;
+      if (ca > cb) { double t = ca; ca = cb; cb = t; }
+      if (ra > rb) { double t = ra; ra = rb; rb = t; }
+      // 1-cell margin; clip in double first (coordinates may be far off the raster)
+      double clo = fmax(floor(ca) - 1.0, 0.0), chi = fmin(floor(cb) + 1.0, (double)(rp.cols - 1));
+      double rlo = fmax(floor(ra) - 1.0, (double)rp.row0);
+      double rhi = fmin(floor(rb) + 1.0, (double)(rp.row0 + rp.nrows - 1));
+      if (clo <= chi && rlo <= rhi) {
+        m.x = (int)((int64_t)clo / rp.T);
+        m.y = (int)((int64_t)chi / rp.T);
+        m.z = (int)((int64_t)rlo / rp.T);
+        m.w = (int)((int64_t)rhi / rp.T);
+        nc = (int64_t)(m.y - m.x + 1) * (m.w - m.z + 1);
+        nb = m.w - m.z + 1;
+      }
+    }
+    mbb[k] = m;
+    ncand[k] = nc;
+    nband[k] = nb;
+  }
+}
+
+__global__ void k_band_count(const int2* __restrict__ erows, const int32_t* __restrict__ epoly, int V, int T,
+                             const int4* __restrict__ mbb, const int64_t* __restrict__ band_base,
+                             int32_t* __restrict__ band_cnt) {
+  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    const int2 rr = erows[v];
+    if (rr.x >= rr.y) continue;
+    const int k = epoly[v];
+    const int4 m = mbb[k];
+    if (m.x > m.y) continue;
+    const int64_t bb = band_base[k];
+    for (int tr = rr.x / T; tr <= (rr.y - 1) / T; ++tr) atomicAdd(&band_cnt[bb + tr - m.z], 1);
+  }
+}
+
+__global__ void k_band_fill(const int2* __restrict__ erows, const int32_t* __restrict__ epoly, int V, int T,
+                            const int4* __restrict__ mbb, const int64_t* __restrict__ band_base,
+                            int32_t* __restrict__ band_cur, int32_t* __restrict__ band_edges) {
+  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    const int2 rr = erows[v];
+    if (rr.x >= rr.y) continue;
+    const int k = epoly[v];
+    const int4 m = mbb[k];
+    if (m.x > m.y) continue;
+    const int64_t bb = band_base[k];
+    for (int tr = rr.x / T; tr <= (rr.y - 1) / T; ++tr) {
+      const int pos = atomicAdd(&band_cur[bb + tr - m.z], 1);
+      band_edges[pos] = v;
+    }
+  }
+}
+
+// Mark INTERSECT: every tile whose cell rectangle comes within one cell of the edge's bounding
+// box (x AND y extent — an edge lying between two centre rows straddles none of them but still
+// separates them).  A tile touched by no edge box is crossed by no part of the boundary, so the
+// exact parity is constant on it, and every straddling edge is >= 1 cell left/right of its
+// centres, so the computed parity equals the exact one at every centre.
+// class: 0 = not yet classified, 1 = inside, 2 = intersect, 3 = outside.
+__global__ void k_mark(const Edge* __restrict__ edges, const int32_t* __restrict__ epoly, int V, Geo g,
+                       RasterP rp, const int4* __restrict__ mbb, const int64_t* __restrict__ cand_off,
+                       uint8_t* __restrict__ cls) {
+  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    const int k = epoly[v];
+    const int4 m = mbb[k];
+    if (m.x > m.y) continue;
+    const Edge e = edges[v];
+    double ca = (fmin(e.xa, e.xb) - g.gt0) / g.gt1, cb = (fmax(e.xa, e.xb) - g.gt0) / g.gt1;
+    if (ca > cb) { double t = ca; ca = cb; cb = t; }
+    double ra = (e.ya - g.gt3) / g.gt5, rb = (e.yb - g.gt3) / g.gt5;
+    if (ra > rb) { double t = ra; ra = rb; rb = t; }
+    const double clo = fmax(floor(ca) - 1.0, (double)m.x * rp.T);
+    const double chi = fmin(floor(cb) + 1.0, (double)(m.y + 1) * rp.T - 1.0);
+    const double rlo = fmax(floor(ra) - 1.0, (double)m.z * rp.T);
+    const double rhi = fmin(floor(rb) + 1.0, (double)(m.w + 1) * rp.T - 1.0);
+    if (clo > chi || rlo > rhi) continue;
+    const int tc_lo = (int)((int64_t)clo / rp.T), tc_hi = (int)((int64_t)chi / rp.T);
+    const int tr_lo = (int)((int64_t)rlo / rp.T), tr_hi = (int)((int64_t)rhi / rp.T);
+    const int wk = m.y - m.x + 1;
+    const int64_t base = cand_off[k];
+    for (int tr = tr_lo; tr <= tr_hi; ++tr)
+      for (int tc = tc_lo; tc <= tc_hi; ++tc) cls[base + (int64_t)(tr - m.z) * wk + (tc - m.x)] = 2;
+  }
+}
+
+// One CTA per band (polygon k, tile row tr): classify the unmarked tiles of the row by the exact
+// PIP status of their first cell (r = tr*T, c = tc*T).  For each band edge straddling r the
+// toggled tiles {tc : xc(tc*T) < xi} form a prefix (gt1 > 0) or a suffix (gt1 < 0) of the row,
+// recorded as flips of a difference bitmap D; parity(j) = XOR_{i > j} D[i].
+__global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges, const int2* __restrict__ erows,
+                                                  const int32_t* __restrict__ band_off,
+                                                  const int32_t* __restrict__ band_edges,
+                                                  const int64_t* __restrict__ band_base, int P, Geo g, RasterP rp,
+                                                  const int4* __restrict__ mbb, const int64_t* __restrict__ cand_off,
+                                                  uint8_t* __restrict__ cls, int dwords) {
+  extern __shared__ uint32_t D[];
+  const int64_t band = blockIdx.x;
+  const int k = (int)(upper_bound_i64(band_base, P + 1, band) - 1);
+  const int4 m = mbb[k];
+  const int tr = m.z + (int)(band - band_base[k]);
+  const int wk = m.y - m.x + 1;
+  const int64_t rrep = (int64_t)tr * rp.T;
+  const double yc = row_centre(g, rrep);
+  const bool s = g.gt1 > 0;
+  for (int i = threadIdx.x; i < dwords; i += blockDim.x) D[i] = 0;
+  __syncthreads();
+  const int e0 = band_off[band], e1 = band_off[band + 1];
+  for (int i = e0 + threadIdx.x; i < e1; i += blockDim.x) {
+    const int v = band_edges[i];
+    const int2 rr = erows[v];
+    if (!(rr.x <= rrep && rrep < rr.y)) continue;
+    const Edge e = edges[v];
+    const double xi = intercept(e, yc);
+    // pred(j) = ((xc(c_j) < xi) == s), true on a prefix of j in [0, wk)
+    const double est = ((xi - g.gt0) / g.gt1 - 0.5) / rp.T - (double)m.x;
+    const int64_t jb = first_false(0, wk, clamp_est(est, 0, wk), [&](int64_t j) {
+      return (col_centre(g, (int64_t)(m.x + j) * rp.T) < xi) == s;
+    });
+    if (jb > 0) atomicXor(&D[jb >> 5], 1u << (jb & 31));
+    if (!s) atomicXor(&D[wk >> 5], 1u << (wk & 31));
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t carry = 0;
+    for (int wi = (wk >> 5); wi >= 0; --wi) {
+      uint32_t t = D[wi];
+      t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
+      D[wi] = (t >> 1) ^ (carry ? 0xFFFFFFFFu : 0u);
+      carry ^= (t & 1u);
+    }
+  }
+  __syncthreads();
+  uint8_t* c = cls + cand_off[k] + (int64_t)(tr - m.z) * wk;
+  for (int j = threadIdx.x; j < wk; j += blockDim.x) {
+    if (c[j] == 0) c[j] = ((D[j >> 5] >> (j & 31)) & 1u) ? 1 : 3;
+  }
+}
+
+__global__ void k_force_isect(uint8_t* cls, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    cls[i] = 2;
+}
+
+__global__ void k_flags(const uint8_t* __restrict__ cls, int64_t n, uint64_t* __restrict__ flags) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint8_t c = cls[i];
+    flags[i] = (c == 1 ? 1ull : 0ull) | (c == 2 ? (1ull << 32) : 0ull);
+  }
+}
+
+__global__ void k_compact(const uint8_t* __restrict__ cls, const uint64_t* __restrict__ pos, int64_t n,
+                          const int64_t* __restrict__ cand_off, int P, const int4* __restrict__ mbb, RasterP rp,
+                          int2* __restrict__ inside, int2* __restrict__ isect, int64_t* __restrict__ totals) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint8_t c = cls[i];
+    if (i == n - 1) {
+      const uint64_t tot = pos[i] + ((c == 1) ? 1ull : 0ull) + ((c == 2) ? (1ull << 32) : 0ull);
+      totals[0] = (int64_t)(tot & 0xFFFFFFFFull);
+      totals[1] = (int64_t)(tot >> 32);
+    }
+    if (c != 1 && c != 2) continue;
+    const int k = (int)(upper_bound_i64(cand_off, P + 1, i) - 1);
+    const int4 m = mbb[k];
+    const int wk = m.y - m.x + 1;
+    const int64_t j = i - cand_off[k];
+    const int tr = m.z + (int)(j / wk), tc = m.x + (int)(j % wk);
+    const int tile = (tr - rp.tr0) * rp.TC + tc;
+    const uint64_t p = pos[i];
+    if (c == 1) inside[p & 0xFFFFFFFFull] = make_int2(tile, k);
+    else isect[p >> 32] = make_int2(tile, k);
+  }
+}
+
+__global__ void k_totals1(const int64_t* cand_off, const int64_t* band_base, const int32_t* espan_sum, int P,
+                          int64_t* out) {
+  out[0] = cand_off[P];
+  out[1] = band_base[P];
+  out[2] = espan_sum[0];
+}
+
+static int grid_for(int64_t n, int threads) {
+  int64_t b = (n + threads - 1) / threads;
+  if (b > 148 * 32) b = 148 * 32;
+  if (b < 1) b = 1;
+  return (int)b;
+}
+
+template <class T>
+static cudaError_t excl_scan(Ctx& c, const T* in, T* out, int64_t n) {
+  size_t need = 0;
+  cudaError_t e = cub::DeviceScan::ExclusiveSum(nullptr, need, in, out, (int)n, c.stream);
+  if (e != cudaSuccess) return e;
+  if ((e = c.d_cub.ensure(need)) != cudaSuccess) return e;
+  size_t have = c.d_cub.bytes;
+  c.launches += 2;  // CUB init + scan kernels
+  return cub::DeviceScan::ExclusiveSum(c.d_cub.p, have, in, out, (int)n, c.stream);
+}
+
+}  // namespace zh
+
+#include <cub/device/device_reduce.cuh>
+
+namespace zh {
+
+cudaError_t launch_pairs_phase1(Ctx& c) {
+  cudaError_t e;
+  const int V = c.V, P = c.P;
+  if ((e = c.d_edges.ensure(sizeof(Edge) * (size_t)V)) != cudaSuccess) return e;
+  if ((e = c.d_erows.ensure(sizeof(int2) * (size_t)V)) != cudaSuccess) return e;
+  if ((e = c.d_epoly.ensure(sizeof(int32_t) * (size_t)V)) != cudaSuccess) return e;
+  if ((e = c.d_espan.ensure(sizeof(int32_t) * ((size_t)V + 1))) != cudaSuccess) return e;
+  if ((e = c.d_mbb.ensure(sizeof(int4) * (size_t)P)) != cudaSuccess) return e;
+  if ((e = c.d_ncand.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
+  if ((e = c.d_nband.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
+  if ((e = c.d_cand_off.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
+  if ((e = c.d_band_base.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
+  if ((e = c.d_counts.ensure(sizeof(int64_t) * 8)) != cudaSuccess) return e;
+  const int64_t rA = c.rp.row0, rB = c.rp.row0 + c.rp.nrows;
+  if (V > 0) {
+    k_edges<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), P, c.d_rvo.as<int32_t>(), c.R,
+                                                   c.d_x.as<double>(), c.d_y.as<double>(), V, c.geo, rA, rB,
+                                                   c.rp.T, c.d_edges.as<Edge>(), c.d_erows.as<int2>(),
+                                                   c.d_epoly.as<int32_t>(), c.d_espan.as<int32_t>());
+    c.launches += 1;
+  }
+  // one trailing zero so that the exclusive scans over P + 1 entries end with the totals
+  cudaMemsetAsync(c.d_ncand.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
+  cudaMemsetAsync(c.d_nband.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
+  if (P > 0) {
+    k_mbb<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
+                                   c.d_y.as<double>(), c.geo, c.rp, c.d_mbb.as<int4>(), c.d_ncand.as<int64_t>(),
+                                   c.d_nband.as<int64_t>());
+    c.launches += 1;
+  }
+  if ((e = excl_scan<int64_t>(c, c.d_ncand.as<int64_t>(), c.d_cand_off.as<int64_t>(), P + 1)) != cudaSuccess) return e;
+  if ((e = excl_scan<int64_t>(c, c.d_nband.as<int64_t>(), c.d_band_base.as<int64_t>(), P + 1)) != cudaSuccess) return e;
+  // espan total (int32 is enough: < 2^31 checked on the host afterwards via int64 sum below)
+  int32_t* sum_out = c.d_espan.as<int32_t>() + V;  // scratch slot
+  if (V > 0) {
+    size_t need = 0;
+    if ((e = cub::DeviceReduce::Sum(nullptr, need, c.d_espan.as<int32_t>(), sum_out, V, c.stream)) != cudaSuccess)
+      return e;
+    if ((e = c.d_cub.ensure(need)) != cudaSuccess) return e;
+    size_t have = c.d_cub.bytes;
+    c.launches += 2;  // CUB reduce kernels
+    if ((e = cub::DeviceReduce::Sum(c.d_cub.p, have, c.d_espan.as<int32_t>(), sum_out, V, c.stream)) != cudaSuccess)
+      return e;
+  } else {
+    cudaMemsetAsync(sum_out, 0, sizeof(int32_t), c.stream);
+  }
+  k_totals1<<<1, 1, 0, c.stream>>>(c.d_cand_off.as<int64_t>(), c.d_band_base.as<int64_t>(), sum_out, P,
+                                   c.d_counts.as<int64_t>());
+  c.launches += 1;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pairs_phase2(Ctx& c) {
+  cudaError_t e;
+  const int V = c.V, P = c.P;
+  const int64_t nc = c.n_cand, nb = c.n_bands, ne = c.n_band_entries;
+  if ((e = c.d_band_cnt.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
+  if ((e = c.d_band_off.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
+  if ((e = c.d_band_cur.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
+  if ((e = c.d_band_edges.ensure(sizeof(int32_t) * (size_t)ne)) != cudaSuccess) return e;
+  if ((e = c.d_class.ensure((size_t)nc)) != cudaSuccess) return e;
+  if ((e = c.d_flags.ensure(sizeof(uint64_t) * (size_t)nc)) != cudaSuccess) return e;
+  if ((e = c.d_flag_pos.ensure(sizeof(uint64_t) * (size_t)nc)) != cudaSuccess) return e;
+  // The band (polygon, tile-row) edge lists.
+  cudaMemsetAsync(c.d_band_cnt.p, 0, sizeof(int32_t) * ((size_t)nb + 1), c.stream);
+  if (V > 0 && nb > 0) {
+    k_band_count<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_erows.as<int2>(), c.d_epoly.as<int32_t>(), V, c.rp.T,
+                                                        c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(),
+                                                        c.d_band_cnt.as<int32_t>());
+    c.launches += 1;
+  }
+  if (nb > 0) {
+    if ((e = excl_scan<int32_t>(c, c.d_band_cnt.as<int32_t>(), c.d_band_off.as<int32_t>(), nb + 1)) != cudaSuccess)
+      return e;
+    cudaMemcpyAsync(c.d_band_cur.p, c.d_band_off.p, sizeof(int32_t) * (size_t)nb, cudaMemcpyDeviceToDevice, c.stream);
+    if (V > 0) {
+      k_band_fill<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_erows.as<int2>(), c.d_epoly.as<int32_t>(), V, c.rp.T,
+                                                         c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(),
+                                                         c.d_band_cur.as<int32_t>(), c.d_band_edges.as<int32_t>());
+      c.launches += 1;
+    }
+  }
+  if (nc > 0) {
+    if (c.force_isect) {
+      k_force_isect<<<grid_for(nc, 256), 256, 0, c.stream>>>(c.d_class.as<uint8_t>(), nc);
+      c.launches += 1;
+    } else {
+      cudaMemsetAsync(c.d_class.p, 0, (size_t)nc, c.stream);
+      if (V > 0) {
+        k_mark<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_edges.as<Edge>(), c.d_epoly.as<int32_t>(), V, c.geo,
+                                                      c.rp, c.d_mbb.as<int4>(),
+                                                      c.d_cand_off.as<int64_t>(), c.d_class.as<uint8_t>());
+        c.launches += 1;
+      }
+      const int dwords = c.rp.TC / 32 + 2;
+      k_classify<<<(unsigned)nb, 128, sizeof(uint32_t) * dwords, c.stream>>>(
+          c.d_edges.as<Edge>(), c.d_erows.as<int2>(), c.d_band_off.as<int32_t>(), c.d_band_edges.as<int32_t>(),
+          c.d_band_base.as<int64_t>(), P, c.geo, c.rp, c.d_mbb.as<int4>(), c.d_cand_off.as<int64_t>(),
+          c.d_class.as<uint8_t>(), dwords);
+      c.launches += 1;
+    }
+    k_flags<<<grid_for(nc, 256), 256, 0, c.stream>>>(c.d_class.as<uint8_t>(), nc, c.d_flags.as<uint64_t>());
+    c.launches += 1;
+    if ((e = excl_scan<uint64_t>(c, c.d_flags.as<uint64_t>(), c.d_flag_pos.as<uint64_t>(), nc)) != cudaSuccess)
+      return e;
+    // lists are sized by the candidate count (an upper bound of both)
+    if ((e = c.d_inside.ensure(sizeof(int2) * (size_t)nc)) != cudaSuccess) return e;
+    if ((e = c.d_isect.ensure(sizeof(int2) * (size_t)nc)) != cudaSuccess) return e;
+    k_compact<<<grid_for(nc, 256), 256, 0, c.stream>>>(c.d_class.as<uint8_t>(), c.d_flag_pos.as<uint64_t>(), nc,
+                                                      c.d_cand_off.as<int64_t>(), P, c.d_mbb.as<int4>(), c.rp,
+                                                      c.d_inside.as<int2>(), c.d_isect.as<int2>(),
+                                                      c.d_counts.as<int64_t>() + 4);
+    c.launches += 1;
+  } else {
+    cudaMemsetAsync(c.d_counts.as<int64_t>() + 4, 0, 2 * sizeof(int64_t), c.stream);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace zh

@@ -1,0 +1,193 @@
+// k_pip.cu — step 4: cell-in-polygon test and histogram update for intersecting pairs
+// (§III.D, Fig. 5, pip_test_kernel).
+//
+// For each intersecting (tile, polygon k) pair and each cell of the tile whose centre passes the
+// even-odd ray-crossing test against all rings of k, out[k][bin(v)] += 1.
+//
+// Paper design (prior art): one block per polygon, one thread per cell, and for every cell a loop
+// over ALL polygon vertices in global memory with float coordinates; the histogram update is a
+// non-atomic read-modify-write (a race).  B200 design, bit-identical to the per-cell test:
+//   * one CTA per intersecting pair; only the edges of the pair's band (edges that straddle one
+//     of the tile's centre rows, built in step 2) are visited;
+//   * the crossing test `xc < xi` depends on the cell only through xc, and xc is monotone in the
+//     column, so for each (edge, row) the crossed cells form a prefix (gt1 > 0) or suffix
+//     (gt1 < 0) of the row: the exact boundary column is found with the SAME xc(c) expression
+//     (first_false), and recorded as a flip in a per-row difference bitmap in shared memory;
+//     a suffix-XOR turns it into the per-cell parity (inside) bits.  Work per pair is
+//     O(#(edge,row) crossings + cells) instead of O(cells x edges);
+//   * edges entirely left / right of the tile's centres (with half a cell of margin, far above
+//     the intercept's rounding) skip the division;
+//   * the cells are then streamed exactly like step 1 (16-byte vectors, inside-mask & nodata /
+//     bin mapping, run merging) into a CTA-private shared histogram, flushed once per pair with
+//     one global atomic per non-zero bin (no race).
+#include "zh_ctx.h"
+
+namespace zh {
+
+struct PipP {
+  RasterP rp;
+  Geo g;
+  BinP bp;
+  const int2* isect;
+  const int4* mbb;
+  const int64_t* band_base;
+  const int32_t* band_off;
+  const int32_t* band_edges;
+  const Edge* edges;
+  const int2* erows;
+  void* out;
+  int B_pad;
+  int wpr;  // bitmap words per row = T/32 + 1
+  int rc;   // rows per chunk
+};
+
+__device__ __forceinline__ uint32_t bits8(const uint32_t* __restrict__ row, int wpr, int lc0) {
+  // parity bits of local columns lc0 .. lc0+7 (lc0 may be negative; missing bits -> 0)
+  if (lc0 >= 0) {
+    const int wi = lc0 >> 5, sh = lc0 & 31;
+    uint64_t v = row[wi];
+    if (sh > 24 && wi + 1 < wpr) v |= (uint64_t)row[wi + 1] << 32;
+    return (uint32_t)(v >> sh) & 0xFFu;
+  }
+  return (row[0] << (-lc0)) & 0xFFu;
+}
+
+template <bool kW1, bool kU64>
+__global__ void __launch_bounds__(256) k_pip(PipP p) {
+  extern __shared__ __align__(16) uint32_t sh[];
+  uint32_t* hist = sh;
+  uint32_t* bm = sh + p.B_pad;
+  const RasterP& rp = p.rp;
+  const Geo& g = p.g;
+
+  const int2 pr = p.isect[blockIdx.x];
+  const int tile = pr.x, k = pr.y;
+  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int tr = rp.tr0 + trl;
+  const int64_t r0 = (int64_t)tr * rp.T;
+  const int h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - r0);
+  const int64_t c0 = (int64_t)tc * rp.T;
+  const int w = (int)min((int64_t)rp.T, rp.cols - c0);
+  const int4 m = p.mbb[k];
+  const int64_t band = p.band_base[k] + (tr - m.z);
+  const int e0 = p.band_off[band], e1 = p.band_off[band + 1];
+  const bool s = g.gt1 > 0;
+  // centre-x range of the tile's columns, and half a cell of margin
+  const double xa_t = col_centre(g, c0), xb_t = col_centre(g, c0 + w - 1);
+  const double xlo_t = fmin(xa_t, xb_t), xhi_t = fmax(xa_t, xb_t);
+  const double half = 0.5 * fabs(g.gt1);
+
+  for (int i = threadIdx.x * 4; i < p.B_pad; i += blockDim.x * 4)
+    *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
+
+  const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
+  const int nk = (int)(k1 - k0);
+  const int64_t pitch = rp.pitch;
+
+  for (int cr = 0; cr < h; cr += p.rc) {
+    const int ch = min(p.rc, h - cr);
+    const int64_t rlo = r0 + cr, rhi = rlo + ch;  // global rows of this chunk
+    for (int i = threadIdx.x; i < ch * p.wpr; i += blockDim.x) bm[i] = 0;
+    __syncthreads();
+    // ---- crossings: flips of the difference bitmap
+    for (int i = e0 + threadIdx.x; i < e1; i += blockDim.x) {
+      const int v = p.band_edges[i];
+      const int2 rr = p.erows[v];
+      const int64_t ra = max((int64_t)rr.x, rlo), rb = min((int64_t)rr.y, rhi);
+      if (ra >= rb) continue;
+      const Edge e = p.edges[v];
+      const double exl = fmin(e.xa, e.xb), exh = fmax(e.xa, e.xb);
+      if (exh + half < xlo_t) continue;  // xi < every xc: crosses no cell of the tile
+      if (exl - half > xhi_t) {          // xi > every xc: crosses every cell
+        for (int64_t r = ra; r < rb; ++r) {
+          const int lr = (int)(r - rlo);
+          atomicXor(&bm[lr * p.wpr + (w >> 5)], 1u << (w & 31));
+        }
+        continue;
+      }
+      for (int64_t r = ra; r < rb; ++r) {
+        const double yc = row_centre(g, r);
+        const double xi = intercept(e, yc);
+        const double est = (xi - g.gt0) / g.gt1 - 0.5 - (double)c0;
+        int64_t ei;
+        if (!(est > 0.0)) ei = 0;
+        else if (est > (double)w) ei = w;
+        else ei = (int64_t)ceil(est);
+        const int64_t jb = first_false(0, w, ei, [&](int64_t j) { return (col_centre(g, c0 + j) < xi) == s; });
+        const int lr = (int)(r - rlo);
+        if (jb > 0) atomicXor(&bm[lr * p.wpr + (int)(jb >> 5)], 1u << (jb & 31));
+        if (!s) atomicXor(&bm[lr * p.wpr + (w >> 5)], 1u << (w & 31));
+      }
+    }
+    __syncthreads();
+    // ---- suffix XOR: parity(lc) = XOR_{j > lc} D[j]
+    for (int lr = threadIdx.x; lr < ch; lr += blockDim.x) {
+      uint32_t* row = bm + lr * p.wpr;
+      uint32_t carry = 0;
+      for (int wi = p.wpr - 1; wi >= 0; --wi) {
+        uint32_t t = row[wi];
+        t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
+        row[wi] = (t >> 1) ^ (carry ? 0xFFFFFFFFu : 0u);
+        carry ^= (t & 1u);
+      }
+    }
+    __syncthreads();
+    // ---- cells: stream the chunk's rows, count inside cells
+    const int16_t* base = rp.data + (rlo - rp.row0) * pitch + k0 * 8;
+    for (int idx = threadIdx.x; idx < ch * nk; idx += blockDim.x) {
+      const int lr = idx / nk, kk = idx - lr * nk;
+      const int64_t cs = (k0 + kk) * 8;
+      uint32_t valid = 0xFFu;
+      if (cs < c0) valid &= (0xFFu << (int)(c0 - cs)) & 0xFFu;
+      if (cs + 8 > c0 + w) valid &= 0xFFu >> (int)(cs + 8 - (c0 + w));
+      valid &= bits8(bm + lr * p.wpr, p.wpr, (int)(cs - c0));
+      if (!valid) continue;
+      const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
+      count8<kW1>(hist, q, valid, p.bp);
+    }
+    __syncthreads();
+  }
+  // ---- flush the pair's histogram
+  const int nbins = p.bp.nbins;
+  const int64_t orow = (int64_t)k * nbins;
+  for (int b = threadIdx.x; b < nbins; b += blockDim.x) {
+    const uint32_t v = hist[b];
+    if (v) {
+      if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(p.out) + orow + b, (unsigned long long)v);
+      else atomicAdd(reinterpret_cast<uint32_t*>(p.out) + orow + b, v);
+    }
+  }
+}
+
+cudaError_t launch_pip(Ctx& c) {
+  if (c.n_isect == 0) return cudaSuccess;
+  PipP p;
+  p.rp = c.rp;
+  p.g = c.geo;
+  p.bp = c.bp;
+  p.isect = c.d_isect.as<int2>();
+  p.mbb = c.d_mbb.as<int4>();
+  p.band_base = c.d_band_base.as<int64_t>();
+  p.band_off = c.d_band_off.as<int32_t>();
+  p.band_edges = c.d_band_edges.as<int32_t>();
+  p.edges = c.d_edges.as<Edge>();
+  p.erows = c.d_erows.as<int2>();
+  p.out = c.d_out;
+  p.B_pad = c.B_pad;
+  p.wpr = c.rp.T / 32 + 1;
+  const int bm_budget_words = 8192;  // 32 KB of parity bitmap per CTA
+  p.rc = bm_budget_words / p.wpr;
+  if (p.rc < 1) p.rc = 1;
+  if (p.rc > c.rp.T) p.rc = c.rp.T;
+  const size_t smem = (size_t)c.B_pad * 4 + (size_t)p.rc * p.wpr * 4;
+  const int threads = 256;
+  void (*k)(PipP);
+  if (c.bp.width == 1) k = c.out_u64 ? k_pip<true, true> : k_pip<true, false>;
+  else k = c.out_u64 ? k_pip<false, true> : k_pip<false, false>;
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<(unsigned)c.n_isect, threads, smem, c.stream>>>(p);
+  c.launches += 1;
+  return cudaGetLastError();
+}
+
+}  // namespace zh

@@ -1,0 +1,400 @@
+// zh_api.cu — the C ABI of libzh (include/zh.h): validation, context lifetime, step orchestration.
+#include <math.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <new>
+#include <vector>
+
+#include "../../include/zh.h"
+#include "zh_ctx.h"
+
+using zh::Ctx;
+
+static thread_local char g_err[512] = "";
+
+static zh_status fail(zh_status s, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+  return s;
+}
+
+static zh_status cuda_fail(cudaError_t e, const char* where) {
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    return fail(ZH_ERR_OOM, "%s: out of device memory", where);
+  }
+  return fail(ZH_ERR_CUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+#define ZH_CU(call, where)                              \
+  do {                                                  \
+    cudaError_t _e = (call);                            \
+    if (_e != cudaSuccess) return cuda_fail(_e, where); \
+  } while (0)
+
+static Ctx* C(zh_ctx c) { return reinterpret_cast<Ctx*>(c); }
+
+extern "C" const char* zh_last_error(void) { return g_err; }
+extern "C" int32_t zh_abi_version(void) { return ZH_ABI_VERSION; }
+
+static const int32_t kMaxBins = 49152;  // shared-memory histogram limit (192 KB per CTA)
+
+static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bins* b, const zh_options* o) {
+  if (!r || !p || !b || !o) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  if (r->rows < 1 || r->cols < 1) return fail(ZH_ERR_INVALID_ARG, "raster rows/cols must be >= 1");
+  if (r->pitch < r->cols) return fail(ZH_ERR_INVALID_ARG, "pitch (%lld) < cols (%lld)", (long long)r->pitch,
+                                      (long long)r->cols);
+  if (r->row0 < 0 || r->nrows < 0 || r->row0 + r->nrows > r->rows)
+    return fail(ZH_ERR_INVALID_ARG, "shard rows [row0, row0+nrows) outside the raster");
+  if (o->tile < 1) return fail(ZH_ERR_INVALID_ARG, "tile must be >= 1");
+  if (r->row0 % o->tile != 0) return fail(ZH_ERR_INVALID_ARG, "row0 must be a multiple of the tile size");
+  for (int i = 0; i < 6; ++i)
+    if (!isfinite(r->gt[i])) return fail(ZH_ERR_INVALID_ARG, "geotransform must be finite");
+  if (r->gt[2] != 0.0 || r->gt[4] != 0.0) return fail(ZH_ERR_UNSUPPORTED, "rotated geotransforms are not supported");
+  if (r->gt[1] == 0.0 || r->gt[5] == 0.0) return fail(ZH_ERR_INVALID_ARG, "gt[1] and gt[5] must be nonzero");
+  if (r->nrows > 0 && !r->data) return fail(ZH_ERR_INVALID_ARG, "raster data is NULL");
+  if (!r->on_host) {
+    if (((uintptr_t)r->data & 15u) != 0) return fail(ZH_ERR_INVALID_ARG, "device raster must be 16-byte aligned");
+    if (r->pitch % 8 != 0) return fail(ZH_ERR_INVALID_ARG, "device raster pitch must be a multiple of 8");
+  }
+  if (r->rows >= (1ll << 31) || r->cols >= (1ll << 31)) return fail(ZH_ERR_UNSUPPORTED, "raster dimension >= 2^31");
+  if (b->nbins < 1 || b->nbins > kMaxBins) return fail(ZH_ERR_INVALID_ARG, "nbins must be in [1, %d]", kMaxBins);
+  if (b->width < 1) return fail(ZH_ERR_INVALID_ARG, "width must be >= 1");
+  if (b->lo > (1 << 30) || b->lo < -(1 << 30)) return fail(ZH_ERR_INVALID_ARG, "|lo| must be <= 2^30");
+  if (p->n_poly < 0 || p->n_ring < 0 || p->n_vert < 0) return fail(ZH_ERR_INVALID_ARG, "negative polygon counts");
+  if (p->n_vert >= (1ll << 31) - 1 || p->n_ring >= (1ll << 31) - 1 || p->n_poly >= (1ll << 31) - 1)
+    return fail(ZH_ERR_UNSUPPORTED, "more than 2^31 vertices/rings/polygons");
+  if (!p->poly_ring_off || !p->ring_vert_off) return fail(ZH_ERR_INVALID_ARG, "null offset array");
+  if (p->n_vert > 0 && (!p->x || !p->y)) return fail(ZH_ERR_INVALID_ARG, "null coordinate array");
+  if (p->poly_ring_off[0] != 0 || p->poly_ring_off[p->n_poly] != p->n_ring)
+    return fail(ZH_ERR_INVALID_ARG, "poly_ring_off must start at 0 and end at n_ring");
+  for (int64_t i = 0; i < p->n_poly; ++i)
+    if (p->poly_ring_off[i + 1] < p->poly_ring_off[i])
+      return fail(ZH_ERR_INVALID_ARG, "poly_ring_off not non-decreasing at %lld", (long long)i);
+  if (p->ring_vert_off[0] != 0 || p->ring_vert_off[p->n_ring] != p->n_vert)
+    return fail(ZH_ERR_INVALID_ARG, "ring_vert_off must start at 0 and end at n_vert");
+  for (int64_t i = 0; i < p->n_ring; ++i)
+    if (p->ring_vert_off[i + 1] < p->ring_vert_off[i])
+      return fail(ZH_ERR_INVALID_ARG, "ring_vert_off not non-decreasing at %lld", (long long)i);
+  double amax = 0.0;
+  for (int64_t i = 0; i < p->n_vert; ++i) {
+    if (!isfinite(p->x[i]) || !isfinite(p->y[i])) return fail(ZH_ERR_INVALID_ARG, "non-finite vertex %lld", (long long)i);
+    amax = std::max(amax, std::max(fabs(p->x[i]), fabs(p->y[i])));
+  }
+  amax = std::max(amax, std::max(fabs(r->gt[0]), fabs(r->gt[3])));
+  amax = std::max(amax, std::max(fabs(r->gt[0] + (double)r->cols * r->gt[1]), fabs(r->gt[3] + (double)r->rows * r->gt[5])));
+  // The classification proof and the quick left/right edge tests need the cell size to dwarf the
+  // rounding of coordinates: |gt1|, |gt5| >= 2^-30 * max |coordinate|.
+  const double lim = ldexp(amax, -30);
+  if (fabs(r->gt[1]) < lim || fabs(r->gt[5]) < lim)
+    return fail(ZH_ERR_UNSUPPORTED, "cell size too small relative to the coordinate magnitude");
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygons* p, const zh_bins* b,
+                               const zh_options* o) {
+  if (!out) return fail(ZH_ERR_INVALID_ARG, "out is NULL");
+  zh_status st = validate(r, p, b, o);
+  if (st != ZH_OK) return st;
+  const int64_t T = o->tile;
+  const int64_t TC = (r->cols + T - 1) / T;
+  const int64_t tr0 = r->row0 / T;
+  const int64_t TRn = (r->nrows + T - 1) / T;
+  const int64_t n_tiles = TC * TRn;
+  if (n_tiles >= (1ll << 31) || TC >= (1ll << 31)) return fail(ZH_ERR_UNSUPPORTED, "more than 2^31 tiles");
+  if (!o->out_u64) {
+    // uint32 output: a polygon's count is bounded by the cells of its MBB
+    for (int64_t k = 0; k < p->n_poly; ++k) {
+      int64_t vb = p->ring_vert_off[p->poly_ring_off[k]], ve = p->ring_vert_off[p->poly_ring_off[k + 1]];
+      if (ve <= vb) continue;
+      double xmn = INFINITY, xmx = -INFINITY, ymn = INFINITY, ymx = -INFINITY;
+      for (int64_t i = vb; i < ve; ++i) {
+        xmn = std::min(xmn, p->x[i]); xmx = std::max(xmx, p->x[i]);
+        ymn = std::min(ymn, p->y[i]); ymx = std::max(ymx, p->y[i]);
+      }
+      double wc = std::min((xmx - xmn) / fabs(r->gt[1]) + 3.0, (double)r->cols);
+      double hc = std::min((ymx - ymn) / fabs(r->gt[5]) + 3.0, (double)r->nrows);
+      if (wc * hc >= 4294967295.0)
+        return fail(ZH_ERR_OVERFLOW, "polygon %lld may hold >= 2^32 cells; use out_u64 = 1", (long long)k);
+    }
+  }
+
+  Ctx* c = new (std::nothrow) Ctx();
+  if (!c) return fail(ZH_ERR_OOM, "host allocation failed");
+  c->rp.data = r->data;
+  c->rp.rows = r->rows;
+  c->rp.cols = r->cols;
+  c->rp.pitch = r->pitch;
+  c->rp.row0 = r->row0;
+  c->rp.nrows = r->nrows;
+  c->rp.T = (int32_t)T;
+  c->rp.TC = (int32_t)TC;
+  c->rp.tr0 = (int32_t)tr0;
+  c->rp.TRn = (int32_t)TRn;
+  c->geo = zh::Geo{r->gt[0], r->gt[1], r->gt[3], r->gt[5]};
+  c->on_host = r->on_host != 0;
+  c->host_data = r->on_host ? r->data : nullptr;
+  c->bp = zh::BinP{b->lo, b->width, b->nbins, b->use_nodata ? 1 : 0, b->nodata, b->oor_drop ? 1 : 0};
+  c->B_pad = (b->nbins + 3) & ~3;
+  c->out_u64 = o->out_u64 ? 1 : 0;
+  c->force_isect = o->force_isect ? 1 : 0;
+  c->stream = (cudaStream_t)o->stream;
+  c->n_tiles = n_tiles;
+  c->P = (int32_t)p->n_poly;
+  c->R = (int32_t)p->n_ring;
+  c->V = (int32_t)p->n_vert;
+
+  auto cleanup_fail = [&](zh_status s) {
+    zh_destroy(reinterpret_cast<zh_ctx>(c));
+    return s;
+  };
+  cudaError_t e;
+  // polygons: int32 offsets + coordinates, copied H2D on the stream
+  std::vector<int32_t> pro(p->n_poly + 1), rvo(p->n_ring + 1);
+  for (int64_t i = 0; i <= p->n_poly; ++i) pro[i] = (int32_t)p->poly_ring_off[i];
+  for (int64_t i = 0; i <= p->n_ring; ++i) rvo[i] = (int32_t)p->ring_vert_off[i];
+  if ((e = c->d_pro.ensure(pro.size() * 4)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
+  if ((e = c->d_rvo.ensure(rvo.size() * 4)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
+  if ((e = c->d_x.ensure((size_t)p->n_vert * 8)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
+  if ((e = c->d_y.ensure((size_t)p->n_vert * 8)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
+  if ((e = cudaMemcpyAsync(c->d_pro.p, pro.data(), pro.size() * 4, cudaMemcpyHostToDevice, c->stream)) ||
+      (e = cudaMemcpyAsync(c->d_rvo.p, rvo.data(), rvo.size() * 4, cudaMemcpyHostToDevice, c->stream)))
+    return cleanup_fail(cuda_fail(e, "zh_create (polygon offsets H2D)"));
+  if (p->n_vert > 0) {
+    if ((e = cudaMemcpyAsync(c->d_x.p, p->x, (size_t)p->n_vert * 8, cudaMemcpyHostToDevice, c->stream)) ||
+        (e = cudaMemcpyAsync(c->d_y.p, p->y, (size_t)p->n_vert * 8, cudaMemcpyHostToDevice, c->stream)))
+      return cleanup_fail(cuda_fail(e, "zh_create (vertices H2D)"));
+  }
+  // per-tile histograms and output
+  if ((e = c->d_tile_hist.ensure((size_t)n_tiles * c->B_pad * 4)) != cudaSuccess)
+    return cleanup_fail(cuda_fail(e, "zh_create (tile histograms)"));
+  const size_t out_bytes = (size_t)p->n_poly * b->nbins * (c->out_u64 ? 8 : 4);
+  if ((e = c->d_out_own.ensure(out_bytes)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (output)"));
+  c->d_out = c->d_out_own.p;
+  if ((e = cudaMemsetAsync(c->d_out, 0, out_bytes, c->stream)) != cudaSuccess)
+    return cleanup_fail(cuda_fail(e, "zh_create"));
+  if (c->on_host) {
+    if ((e = c->raster_dev.ensure((size_t)std::max<int64_t>(r->nrows, 1) * r->pitch * 2 + 16)) != cudaSuccess)
+      return cleanup_fail(cuda_fail(e, "zh_create (device raster copy)"));
+    c->rp.data = c->raster_dev.as<int16_t>();
+    if (r->pitch % 8 != 0) return cleanup_fail(fail(ZH_ERR_INVALID_ARG, "host raster pitch must be a multiple of 8"));
+  }
+  if ((e = cudaHostAlloc((void**)&c->pinned_counts, 8 * sizeof(int64_t), cudaHostAllocDefault)) != cudaSuccess)
+    return cleanup_fail(cuda_fail(e, "zh_create (pinned counters)"));
+  for (int i = 0; i < 8; ++i)
+    if ((e = cudaEventCreate(&c->ev[i])) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (events)"));
+  if ((e = cudaGetLastError()) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
+  *out = reinterpret_cast<zh_ctx>(c);
+  return ZH_OK;
+}
+
+extern "C" void zh_destroy(zh_ctx h) {
+  if (!h) return;
+  Ctx* c = C(h);
+  cudaStreamSynchronize(c->stream);
+  zh::DBuf* bufs[] = {&c->raster_dev, &c->d_pro, &c->d_rvo, &c->d_x, &c->d_y, &c->d_edges, &c->d_erows,
+                      &c->d_epoly, &c->d_espan, &c->d_mbb, &c->d_ncand, &c->d_nband, &c->d_cand_off,
+                      &c->d_band_base, &c->d_band_cnt, &c->d_band_off, &c->d_band_cur, &c->d_band_edges,
+                      &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
+                      &c->d_cub, &c->d_tile_hist, &c->d_out_own};
+  for (auto* b : bufs) b->release();
+  for (int i = 0; i < 8; ++i)
+    if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  if (c->pinned_counts) cudaFreeHost(c->pinned_counts);
+  delete c;
+}
+
+size_t zh::device_bytes(const Ctx& c) {
+  const zh::DBuf* bufs[] = {&c.raster_dev, &c.d_pro, &c.d_rvo, &c.d_x, &c.d_y, &c.d_edges, &c.d_erows,
+                            &c.d_epoly, &c.d_espan, &c.d_mbb, &c.d_ncand, &c.d_nband, &c.d_cand_off,
+                            &c.d_band_base, &c.d_band_cnt, &c.d_band_off, &c.d_band_cur, &c.d_band_edges,
+                            &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
+                            &c.d_cub, &c.d_tile_hist, &c.d_out_own};
+  size_t s = 0;
+  for (auto* b : bufs) s += b->bytes;
+  return s;
+}
+
+static void tic(Ctx* c, int step) {
+  if (c->timing) cudaEventRecord(c->ev[2 * step], c->stream);
+}
+static void toc(Ctx* c, int step) {
+  if (c->timing) cudaEventRecord(c->ev[2 * step + 1], c->stream);
+}
+
+extern "C" zh_status zh_upload_raster(zh_ctx h) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (!c->on_host) return ZH_OK;
+  if (c->rp.nrows > 0)
+    ZH_CU(cudaMemcpyAsync(c->raster_dev.p, c->host_data, (size_t)c->rp.nrows * c->rp.pitch * 2, cudaMemcpyHostToDevice,
+                          c->stream),
+          "zh_upload_raster");
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_tile_hist(zh_ctx h) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  tic(c, 0);
+  ZH_CU(zh::launch_tile_hist(*c), "zh_tile_hist");
+  toc(c, 0);
+  c->have_hist = true;
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  c->have_pairs = false;
+  c->step3_done = false;
+  tic(c, 1);
+  const size_t out_bytes = (size_t)c->P * c->bp.nbins * (c->out_u64 ? 8 : 4);
+  ZH_CU(cudaMemsetAsync(c->d_out, 0, out_bytes, c->stream), "zh_pair_tiles (zero output)");
+  ZH_CU(zh::launch_pairs_phase1(*c), "zh_pair_tiles (phase 1)");
+  ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_counts.p, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
+        "zh_pair_tiles (counts)");
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_pair_tiles (sync 1)");
+  c->n_cand = c->pinned_counts[0];
+  c->n_bands = c->pinned_counts[1];
+  c->n_band_entries = c->pinned_counts[2];
+  if (c->n_cand >= (1ll << 31) || c->n_bands >= (1ll << 31) || c->n_band_entries >= (1ll << 31) ||
+      c->n_band_entries < 0)
+    return fail(ZH_ERR_UNSUPPORTED, "pair lists exceed 2^31 entries");
+  ZH_CU(zh::launch_pairs_phase2(*c), "zh_pair_tiles (phase 2)");
+  ZH_CU(cudaMemcpyAsync(c->pinned_counts + 4, c->d_counts.as<int64_t>() + 4, 2 * sizeof(int64_t),
+                        cudaMemcpyDeviceToHost, c->stream),
+        "zh_pair_tiles (counts)");
+  toc(c, 1);
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_pair_tiles (sync 2)");
+  c->n_inside = c->pinned_counts[4];
+  c->n_isect = c->pinned_counts[5];
+  c->have_pairs = true;
+  if (n_inside) *n_inside = c->n_inside;
+  if (n_isect) *n_isect = c->n_isect;
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_aggregate(zh_ctx h) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (!c->have_pairs || !c->have_hist) return fail(ZH_ERR_STATE, "zh_aggregate needs zh_tile_hist and zh_pair_tiles");
+  if (c->step3_done) return fail(ZH_ERR_STATE, "zh_aggregate already applied since the last zh_pair_tiles");
+  tic(c, 2);
+  ZH_CU(zh::launch_aggregate(*c), "zh_aggregate");
+  toc(c, 2);
+  c->step3_done = true;
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_pip_update(zh_ctx h) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (!c->have_pairs) return fail(ZH_ERR_STATE, "zh_pip_update needs zh_pair_tiles");
+  tic(c, 3);
+  ZH_CU(zh::launch_pip(*c), "zh_pip_update");
+  toc(c, 3);
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_run(zh_ctx h, void* host_out) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  zh_status s;
+  if ((s = zh_upload_raster(h)) != ZH_OK) return s;
+  if ((s = zh_pair_tiles(h, nullptr, nullptr)) != ZH_OK) return s;
+  if ((s = zh_tile_hist(h)) != ZH_OK) return s;
+  if ((s = zh_aggregate(h)) != ZH_OK) return s;
+  if ((s = zh_pip_update(h)) != ZH_OK) return s;
+  if (host_out) {
+    const size_t out_bytes = (size_t)c->P * c->bp.nbins * (c->out_u64 ? 8 : 4);
+    ZH_CU(cudaMemcpyAsync(host_out, c->d_out, out_bytes, cudaMemcpyDeviceToHost, c->stream), "zh_run (D2H)");
+  }
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_run (sync)");
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_output_device(zh_ctx h, void** dptr, int64_t* n) {
+  if (!h || !dptr) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  Ctx* c = C(h);
+  *dptr = c->d_out;
+  if (n) *n = (int64_t)c->P * c->bp.nbins;
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_set_output(zh_ctx h, void* dptr) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (dptr && ((uintptr_t)dptr & 7u)) return fail(ZH_ERR_INVALID_ARG, "output buffer must be 8-byte aligned");
+  c->d_out = dptr ? dptr : c->d_out_own.p;
+  c->have_pairs = false;  // the new buffer must be zeroed by zh_pair_tiles before accumulation
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_copy_tile_hist(zh_ctx h, uint32_t* host, int64_t n_elems) {
+  if (!h || !host) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  Ctx* c = C(h);
+  if (n_elems < c->n_tiles * c->bp.nbins) return fail(ZH_ERR_INVALID_ARG, "host buffer too small");
+  if (c->n_tiles == 0) return ZH_OK;
+  ZH_CU(cudaMemcpy2DAsync(host, (size_t)c->bp.nbins * 4, c->d_tile_hist.p, (size_t)c->B_pad * 4,
+                          (size_t)c->bp.nbins * 4, (size_t)c->n_tiles, cudaMemcpyDeviceToHost, c->stream),
+        "zh_copy_tile_hist");
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_copy_tile_hist");
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_copy_pairs(zh_ctx h, int32_t* inside, int32_t* isect) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (!c->have_pairs) return fail(ZH_ERR_STATE, "zh_copy_pairs needs zh_pair_tiles");
+  if (inside && c->n_inside)
+    ZH_CU(cudaMemcpyAsync(inside, c->d_inside.p, (size_t)c->n_inside * 8, cudaMemcpyDeviceToHost, c->stream),
+          "zh_copy_pairs");
+  if (isect && c->n_isect)
+    ZH_CU(cudaMemcpyAsync(isect, c->d_isect.p, (size_t)c->n_isect * 8, cudaMemcpyDeviceToHost, c->stream),
+          "zh_copy_pairs");
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_copy_pairs");
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
+  if (!h || !s) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  Ctx* c = C(h);
+  s->n_tiles = c->n_tiles;
+  s->n_candidates = c->n_cand;
+  s->n_inside = c->n_inside;
+  s->n_isect = c->n_isect;
+  s->n_band_entries = c->n_band_entries;
+  s->n_edges = c->V;
+  s->device_bytes = (int64_t)zh::device_bytes(*c);
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_set_timing(zh_ctx h, int32_t enable) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  C(h)->timing = enable != 0;
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_get_step_ms(zh_ctx h, float* ms4) {
+  if (!h || !ms4) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  Ctx* c = C(h);
+  if (!c->timing) return fail(ZH_ERR_STATE, "timing is disabled");
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_step_ms");
+  for (int i = 0; i < 4; ++i) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, c->ev[2 * i], c->ev[2 * i + 1]) != cudaSuccess) {
+      cudaGetLastError();
+      ms = -1.f;
+    }
+    ms4[i] = ms;
+  }
+  return ZH_OK;
+}
+
+extern "C" int64_t zh_launch_count(zh_ctx h) { return h ? C(h)->launches : 0; }

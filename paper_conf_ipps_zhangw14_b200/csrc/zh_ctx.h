@@ -1,0 +1,81 @@
+// zh_ctx.h — host-side context of libzh and the launchers of its kernels (internal).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "zh_internal.cuh"
+
+namespace zh {
+
+// Grow-only device buffer owned by the context.
+struct DBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  cudaError_t ensure(size_t need) {
+    if (need <= bytes && p) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+    if (need == 0) need = 16;
+    cudaError_t e = cudaMalloc(&p, need);
+    if (e == cudaSuccess) bytes = need;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+  }
+  template <class T>
+  T* as() const { return reinterpret_cast<T*>(p); }
+};
+
+struct Ctx {
+  // raster shard
+  RasterP rp;
+  Geo geo;
+  const int16_t* host_data = nullptr;  // on_host rasters: borrowed host pointer
+  bool on_host = false;
+  DBuf raster_dev;                     // on_host rasters: device copy of the shard
+  // bins / options
+  BinP bp;
+  int32_t B_pad = 0;
+  int32_t out_u64 = 1;
+  int32_t force_isect = 0;
+  cudaStream_t stream = nullptr;
+  // polygons (device)
+  int32_t P = 0, R = 0, V = 0;
+  DBuf d_pro, d_rvo, d_x, d_y;
+  // step 2 products
+  DBuf d_edges, d_erows, d_epoly, d_espan, d_mbb, d_ncand, d_nband, d_cand_off, d_band_base;
+  DBuf d_band_cnt, d_band_off, d_band_cur, d_band_edges, d_class, d_flags, d_flag_pos;
+  DBuf d_inside, d_isect, d_counts, d_cub;
+  int64_t n_cand = 0, n_bands = 0, n_band_entries = 0, n_inside = 0, n_isect = 0;
+  // step 1 product and output
+  DBuf d_tile_hist;
+  DBuf d_out_own;
+  void* d_out = nullptr;  // own or borrowed
+  int64_t n_tiles = 0;
+  // state
+  bool have_hist = false, have_pairs = false, step3_done = false;
+  // timing
+  bool timing = false;
+  cudaEvent_t ev[8] = {};
+  float step_ms[4] = {0, 0, 0, 0};
+  int64_t launches = 0;
+  int64_t host_count_buf[4] = {0, 0, 0, 0};
+  int64_t* pinned_counts = nullptr;
+};
+
+// kernels / launchers (k_*.cu)
+cudaError_t launch_tile_hist(Ctx& c);
+cudaError_t launch_pairs_phase1(Ctx& c);   // edges, MBBs, scans, count totals -> d_counts
+cudaError_t launch_pairs_phase2(Ctx& c);   // bands, marking, classification, compaction
+cudaError_t launch_aggregate(Ctx& c);
+cudaError_t launch_pip(Ctx& c);
+
+size_t device_bytes(const Ctx& c);
+
+}  // namespace zh

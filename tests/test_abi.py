@@ -1,0 +1,126 @@
+"""CPU-side checks of the boundary: libzh builds for sm_100a, loads, exports every symbol zh.h
+declares, and rejects malformed input without touching a GPU (validation happens before any
+CUDA call)."""
+import ctypes
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "zh.h")).read()
+    return sorted(set(re.findall(r"^\s*(?:zh_status|void|const char\*|int32_t|int64_t)\s+(zh_\w+)\s*\(", src, re.M)))
+
+
+def test_header_declares_the_north_star_calls():
+    names = _declared()
+    for n in ["zh_create", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update", "zh_run",
+              "zh_output_device", "zh_last_error", "zh_destroy"]:
+        assert n in names
+
+
+def test_library_exports_every_declared_symbol():
+    from paper_conf_ipps_zhangw14_b200 import _build
+    lib = _build.build()
+    out = subprocess.run(["nm", "-D", "--defined-only", lib], capture_output=True, text=True, check=True).stdout
+    exported = set(re.findall(r"\bT (zh_\w+)", out))
+    missing = [n for n in _declared() if n not in exported]
+    assert not missing, missing
+    from paper_conf_ipps_zhangw14_b200 import zh
+    assert set(zh.EXPORTS) == set(_declared())
+    assert zh.LIB.zh_abi_version() == 1
+
+
+def test_library_is_sm100a_sass():
+    from paper_conf_ipps_zhangw14_b200 import _build
+    lib = _build.build()
+    out = subprocess.run(["cuobjdump", "--list-elf", lib], capture_output=True, text=True, check=True).stdout
+    assert "sm_100a" in out
+
+
+def test_pip_predicate_has_no_contracted_fma():
+    """The intercept / centre expressions must be separate DMUL/DADD (R7).  DFMA may only appear
+    inside the IEEE division routine; check that every DFMA sits in a division sequence by
+    verifying the kernel's DFMA count equals that of a kernel with only the divisions."""
+    from paper_conf_ipps_zhangw14_b200 import _build
+    lib = _build.build()
+    sass = subprocess.run(["cuobjdump", "-sass", "-fun", "_ZN2zh5k_pipILb1ELb1EEEvNS_4PipPE", lib],
+                          capture_output=True, text=True, check=True).stdout
+    assert "DMUL" in sass and "DADD" in sass
+    # the division routine's DFMAs follow an MUFU.RCP64H; no DFMA may consume the centre/intercept
+    # operands directly — weak check: DFMA count is bounded by the number of reciprocal sequences
+    n_dfma = sass.count("DFMA")
+    n_rcp = sass.count("MUFU.RCP64H")
+    assert n_rcp >= 1
+    assert n_dfma <= 8 * n_rcp + 8
+
+
+def _mk(lib_zh, **over):
+    zh = lib_zh
+    r = zh.zh_raster()
+    buf = np.zeros((16, 16), np.int16)
+    r.data = buf.ctypes.data
+    r.rows, r.cols, r.pitch, r.row0, r.nrows = 16, 16, 16, 0, 16
+    r.gt = (ctypes.c_double * 6)(0, 1, 0, 16, 0, -1)
+    r.on_host = 1
+    pro = np.array([0, 1], np.int64)
+    rvo = np.array([0, 3], np.int64)
+    x = np.array([0.0, 8, 0])
+    y = np.array([0.0, 0, 8])
+    p = zh.zh_polygons(1, 1, 3, pro.ctypes.data, rvo.ctypes.data, x.ctypes.data, y.ctypes.data)
+    b = zh.zh_bins(0, 1, 16, 0, 0, 0)
+    o = zh.zh_options(4, 1, 0, 0, None)
+    for k, v in over.items():
+        obj, field = k.split("__")
+        target = {"r": r, "p": p, "b": b, "o": o}[obj]
+        setattr(target, field, v)
+    return r, p, b, o, (buf, pro, rvo, x, y)
+
+
+@pytest.mark.parametrize("over,status", [
+    ({"o__tile": 0}, 1), ({"b__nbins": 0}, 1), ({"b__width": 0}, 1), ({"r__pitch": 8}, 1),
+    ({"r__row0": 3, "r__nrows": 8}, 1), ({"r__nrows": 20}, 1), ({"b__nbins": 1 << 20}, 1),
+])
+def test_create_rejects_malformed_input(over, status):
+    from paper_conf_ipps_zhangw14_b200 import zh
+    r, p, b, o, keep = _mk(zh, **over)
+    h = ctypes.c_void_p()
+    st = zh.LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o))
+    assert st == status
+    assert h.value is None
+    assert zh.LIB.zh_last_error()
+
+
+def test_create_rejects_rotation_nan_and_bad_offsets():
+    from paper_conf_ipps_zhangw14_b200 import zh
+    r, p, b, o, keep = _mk(zh)
+    r.gt = (ctypes.c_double * 6)(0, 1, 0.1, 16, 0, -1)
+    h = ctypes.c_void_p()
+    assert zh.LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)) == 2
+    r, p, b, o, keep = _mk(zh)
+    keep[3][1] = np.nan
+    assert zh.LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)) == 1
+    r, p, b, o, keep = _mk(zh)
+    keep[2][1] = 5  # ring_vert_off end != n_vert
+    assert zh.LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)) == 1
+    # uint32 output with a polygon whose MBB could exceed 2^32 cells
+    r, p, b, o, keep = _mk(zh)
+    r.rows, r.cols, r.nrows = 100000, 100000, 100000
+    keep[3][:] = [0, 1e6, 0]
+    keep[4][:] = [0, 0, -1e6]
+    r.pitch = 100000
+    o.out_u64 = 0
+    assert zh.LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)) == 5
+
+
+def test_null_context_calls_fail_cleanly():
+    from paper_conf_ipps_zhangw14_b200 import zh
+    for f in ["zh_tile_hist", "zh_aggregate", "zh_pip_update", "zh_upload_raster"]:
+        assert getattr(zh.LIB, f)(None) == 1
+    assert zh.LIB.zh_run(None, None) == 1
+    zh.LIB.zh_destroy(None)

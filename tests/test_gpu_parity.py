@@ -1,0 +1,257 @@
+"""GPU parity: libzh (through the C ABI) vs the CPU oracle, element by element, bit-exact.
+
+Inputs come from synth/ (seeded; the device raster is generated on the GPU and checked equal to
+the host raster the oracle reads).  The oracle never sees anything computed by libzh.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from synth.configs import TINY, TINY_LONLAT
+from synth.dem import KIND_LINMOD, DemSpec, fill_device, fill_host
+from synth.polygons import from_rings
+
+pytestmark = pytest.mark.gpu
+
+
+def _zh():
+    from paper_conf_ipps_zhangw14_b200 import zh
+    return zh
+
+
+def device_raster(spec, rows, cols, row0=0, nrows=None, pitch=None, gcols=None):
+    import torch
+    nrows = rows - row0 if nrows is None else nrows
+    pitch = pitch or ((cols + 7) // 8 * 8)
+    t = torch.full((nrows, pitch), 12345, dtype=torch.int16, device="cuda")
+    fill_device(spec, gcols or cols, t.data_ptr(), row0, 0, nrows, cols, pitch,
+                torch.cuda.current_stream().cuda_stream)
+    return t
+
+
+def gpu_hist(t, gt, P, nbins, tile, cols, rows=None, row0=0, **kw):
+    zh = _zh()
+    with zh.ZonalHistogram(t, gt, P, nbins, tile=tile, cols=cols, rows=rows, row0=row0, **kw) as z:
+        return z.run()
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    cfg = TINY
+    P = cfg.polygons()
+    R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
+    bins = oracle.make_bins(cfg.nbins, nodata=cfg.nodata)
+    H = oracle.o0(R, cfg.gt, P, bins)
+    return cfg, P, R, H
+
+
+def test_device_generator_matches_host(tiny, cuda_device):
+    cfg, P, R, _ = tiny
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    assert (t.cpu().numpy()[:, :cfg.cols] == R).all()
+
+
+@pytest.mark.parametrize("out_u64", [True, False])
+def test_tiny_bit_exact(tiny, cuda_device, out_u64):
+    cfg, P, R, H = tiny
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    G = gpu_hist(t, cfg.gt, P, cfg.nbins, cfg.tile, cfg.cols, nodata=cfg.nodata, out_u64=out_u64)
+    assert (G.astype(np.uint64) == H).all()
+
+
+@pytest.mark.parametrize("tile", [1, 5, 8, 13, 64, 100, 128, 256, 360, 1000, 1024, 2048])
+def test_tiny_tile_size_invariance(tiny, cuda_device, tile):
+    cfg, P, R, H = tiny
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    G = gpu_hist(t, cfg.gt, P, cfg.nbins, tile, cfg.cols, nodata=cfg.nodata)
+    assert (G == H).all()
+
+
+def test_force_all_intersect_identical(tiny, cuda_device):
+    cfg, P, R, H = tiny
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    for tile in (64, 128):
+        G = gpu_hist(t, cfg.gt, P, cfg.nbins, tile, cfg.cols, nodata=cfg.nodata, force_isect=True)
+        assert (G == H).all()
+
+
+def test_step1_tile_histograms_vs_bincount(tiny, cuda_device):
+    cfg, P, R, H = tiny
+    zh = _zh()
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    T = 100  # ragged edge tiles, unaligned columns
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=T, cols=cfg.cols, nodata=cfg.nodata) as z:
+        z.zh_tile_hist()
+        th = z.tile_hist_host()
+    TC = (cfg.cols + T - 1) // T
+    for tid in range(th.shape[0]):
+        tr, tc = divmod(tid, TC)
+        blk = R[tr * T:(tr + 1) * T, tc * T:(tc + 1) * T].astype(np.int64).ravel()
+        blk = blk[blk != cfg.nodata]
+        ref = np.bincount(np.clip(blk, 0, cfg.nbins - 1), minlength=cfg.nbins)
+        assert (th[tid] == ref).all(), tid
+
+
+def test_step2_classification_is_sound(tiny, cuda_device):
+    """Inside pairs: every cell centre of the tile is inside (oracle); outside (unlisted) MBB
+    tiles: no centre inside; intersect pairs are whatever is left."""
+    cfg, P, R, H = tiny
+    zh = _zh()
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    T = 64
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=T, cols=cfg.cols, nodata=cfg.nodata) as z:
+        ni, nx = z.zh_pair_tiles()
+        ins, isx = z.pairs_host()
+    assert ni > 0 and nx > 0
+    TC = (cfg.cols + T - 1) // T
+    rr, cc = np.meshgrid(np.arange(cfg.rows), np.arange(cfg.cols), indexing="ij")
+    mem = oracle.membership(rr.ravel(), cc.ravel(), cfg.gt, P).reshape(cfg.rows, cfg.cols, P.n_poly)
+    listed = set()
+    for tile, k in ins:
+        tr, tc = divmod(int(tile), TC)
+        assert mem[tr * T:(tr + 1) * T, tc * T:(tc + 1) * T, k].all()
+        listed.add((int(tile), int(k)))
+    for tile, k in isx:
+        listed.add((int(tile), int(k)))
+    for tid in range(TC * TC):
+        tr, tc = divmod(tid, TC)
+        blk = mem[tr * T:(tr + 1) * T, tc * T:(tc + 1) * T]
+        for k in np.nonzero(blk.reshape(-1, P.n_poly).any(axis=0))[0]:
+            assert (tid, int(k)) in listed
+    # lists sorted by (polygon, tile)
+    for L in (ins, isx):
+        key = L[:, 1].astype(np.int64) * (1 << 32) + L[:, 0]
+        assert (np.diff(key) > 0).all()
+
+
+def test_tiny_lonlat_bit_exact(cuda_device):
+    cfg = TINY_LONLAT
+    P = cfg.polygons()
+    R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata))
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    for tile in (32, 128, 200):
+        assert (gpu_hist(t, cfg.gt, P, cfg.nbins, tile, cfg.cols, nodata=cfg.nodata) == H).all()
+
+
+@pytest.mark.parametrize("flip", ["x", "y", "xy"])
+def test_flipped_geotransforms(tiny, cuda_device, flip):
+    cfg, P, R, _ = tiny
+    gt = list(cfg.gt)
+    if "x" in flip:
+        gt[0], gt[1] = float(cfg.cols), -1.0
+    if "y" in flip:
+        gt[3], gt[5] = 0.0, 1.0
+    H = oracle.o1(R, gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata))
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    for tile in (64, 100):
+        assert (gpu_hist(t, gt, P, cfg.nbins, tile, cfg.cols, nodata=cfg.nodata) == H).all()
+
+
+@pytest.mark.parametrize("lo,width,nbins,drop,nodata", [(0, 1, 256, True, -32768), (-100, 3, 77, False, None),
+                                                         (20, 7, 9, True, -32768), (-20, 1, 300, False, 150)])
+def test_bin_mappings(tiny, cuda_device, lo, width, nbins, drop, nodata):
+    cfg, P, R, _ = tiny
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(nbins, lo=lo, width=width, nodata=nodata, oor_drop=drop))
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    G = gpu_hist(t, cfg.gt, P, nbins, 128, cfg.cols, lo=lo, width=width, nodata=nodata, oor_drop=drop)
+    assert (G == H).all()
+
+
+def test_ragged_raster_and_pitch(cuda_device):
+    """1000 x 1003 raster (cols not a multiple of 8), pitch 1016, tiles 96 and 128 (ragged)."""
+    rows, cols = 1000, 1003
+    gt = (0.0, 1.0, 0.0, float(rows), 0.0, -1.0)
+    spec = DemSpec(seed=21, base=-150, macro_amp=900, fine_amp=200)
+    from synth.polygons import voronoi_tiling
+    P = voronoi_tiling(cols, rows, gt, 12, 5, 22, n_holes=2)
+    R = fill_host(spec, cols, 0, 0, rows, cols)
+    H = oracle.o1(R, gt, P, oracle.make_bins(256, nodata=-32768))
+    t = device_raster(spec, rows, cols, pitch=1016)
+    for tile in (96, 128, 1003):
+        assert (gpu_hist(t, gt, P, 256, tile, cols, nodata=-32768) == H).all()
+
+
+def test_hand_worked_cases_on_gpu(cuda_device):
+    import os
+    import torch
+    gold = os.path.join(os.path.dirname(__file__), "golden", "hand_counts.txt")
+    names, polys, want = [], [], []
+    for line in open(gold):
+        if line.startswith("#") or not line.strip():
+            continue
+        n, rings, c, _ = [f.strip() for f in line.split("|")]
+        rr = []
+        for part in rings.split("/"):
+            pts = [tuple(map(float, p.split(","))) for p in part.split()]
+            rr.append((np.array([p[0] for p in pts]), np.array([p[1] for p in pts])))
+        names.append(n)
+        polys.append(rr)
+        want.append(int(c))
+    P = from_rings(polys)
+    t = torch.zeros((20, 24), dtype=torch.int16, device="cuda")
+    for tile in (1, 3, 4, 8, 24):
+        G = gpu_hist(t, (0.0, 1.0, 0.0, 20.0, 0.0, -1.0), P, 1, tile, 24)
+        assert [int(g) for g in G[:, 0]] == want, (tile, names)
+
+
+def test_degenerate_polygons(cuda_device):
+    cfg = TINY
+    R = fill_host(cfg.dem, cfg.cols, 0, 0, 64, 64)
+    gt = (0.0, 1.0, 0.0, 64.0, 0.0, -1.0)
+    sq = (np.array([5.0, 30, 30, 5]), np.array([5.0, 5, 30, 30]))
+    P = from_rings([[], [(np.array([]), np.array([]))], [(np.array([3.0]), np.array([3.0]))],
+                    [(np.array([3.0, 40]), np.array([3.0, 50]))], [sq],
+                    [(np.append(sq[0], 5.0), np.append(sq[1], 5.0))], [(sq[0] + 1000, sq[1])],
+                    [(np.repeat(sq[0], 2), np.repeat(sq[1], 2))], [(sq[0] - 1000, sq[1] + 1e6)]])
+    H = oracle.o0(R, gt, P, oracle.make_bins(256, nodata=-32768))
+    t = device_raster(cfg.dem, 64, 64, gcols=cfg.cols)
+    for tile in (8, 16, 64):
+        assert (gpu_hist(t, gt, P, 256, tile, 64, nodata=-32768) == H).all()
+    # no polygons at all
+    E = from_rings([])
+    assert gpu_hist(t, gt, E, 256, 16, 64).shape == (0, 256)
+
+
+def test_tile_row_shards_sum_to_whole(tiny, cuda_device):
+    """Shards of whole tile rows (the multi-GPU decomposition) sum to the single-shard result."""
+    cfg, P, R, H = tiny
+    T = 128
+    for nsh in (2, 3, 8):
+        tiles_rows = (cfg.rows + T - 1) // T
+        per = -(-tiles_rows // nsh)
+        acc = np.zeros_like(H)
+        for g in range(nsh):
+            r0 = min(cfg.rows, g * per * T)
+            r1 = min(cfg.rows, (g + 1) * per * T)
+            t = device_raster(cfg.dem, cfg.rows, cfg.cols, row0=r0, nrows=r1 - r0)
+            acc += gpu_hist(t, cfg.gt, P, cfg.nbins, T, cfg.cols, rows=cfg.rows, row0=r0, nodata=cfg.nodata)
+        assert (acc == H).all()
+
+
+def test_host_raster_path(tiny, cuda_device):
+    import torch
+    cfg, P, R, H = tiny
+    pinned = torch.from_numpy(R.copy()).pin_memory()
+    G = gpu_hist(pinned, cfg.gt, P, cfg.nbins, cfg.tile, cfg.cols, nodata=cfg.nodata)
+    assert (G == H).all()
+
+
+def test_overlapping_polygons_and_linear_pattern(cuda_device):
+    """Overlapping polygons count a cell in each; v = (r*cols + c) mod 4093 exercises all bins."""
+    rows, cols = 512, 768
+    gt = (10.0, 0.5, 0.0, 300.0, 0.0, -0.25)
+    spec = DemSpec(kind=KIND_LINMOD, pattern_mod=4093, pattern_off=-7)
+    R = fill_host(spec, cols, 0, 0, rows, cols)
+    rng = np.random.default_rng(5)
+    polys = []
+    for _ in range(40):
+        cx, cy = rng.uniform(10, 394), rng.uniform(172, 300)
+        th = np.sort(rng.uniform(0, 2 * np.pi, 30))
+        rad = rng.uniform(5, 60, 30)
+        polys.append([(cx + rad * np.cos(th), cy + rad * np.sin(th))])
+    P = from_rings(polys)
+    H = oracle.o1(R, gt, P, oracle.make_bins(4096, lo=-7))
+    t = device_raster(spec, rows, cols)
+    for tile in (32, 64, 256):
+        assert (gpu_hist(t, gt, P, 4096, tile, cols, lo=-7) == H).all()
