@@ -1,0 +1,434 @@
+#!/usr/bin/env python
+"""bench.py — zonal histogramming throughput on B200 (raster cells/s, end-to-end), driver contract.
+
+A "step" is one pass of the whole hot path: zh_pair_tiles (step 2, incl.
+zeroing the output), zh_tile_hist (step 1), zh_aggregate (step 3), zh_pip_update (step 4) over
+the CONUS-scale synthetic raster (93,600 x 216,000 int16 = 20.2 G cells, 40.4 GB resident in HBM)
+and ~3,100 jagged county polygons; with N > 1 GPUs each rank holds a strip of whole tile rows
+and the step ends with an NCCL all-reduce of the [n_poly, 5000] uint64 histograms.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config conus] [--impl ours|reference]
+
+value = raster cells of the whole job / device time per step (max over ranks; CUDA events).
+e2e   = the same metric through the public C ABI from HOST buffers: per step zh_create (polygon
+        H2D) + zh_run on a pinned host raster (raster H2D, the four steps, result D2H).
+roofline = the dominant kernel's algorithmic bytes / its CUDA-event time vs measured HBM peak.
+cpu_baseline = the CPU oracle (oracle/, O1 row-hoisted, all host cores) on a bounded row band.
+--impl reference = that oracle as the reference arm (this tier has no reference implementation).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CLOCK_Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+           "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+           "clocks_event_reasons.sw_power_cap")
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.lines: list[str] = []
+        self.proc = None
+        self.t = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={CLOCK_Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            if self.t is not None:
+                self.t.join(timeout=2)
+
+    def summary(self) -> dict:
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def measured_peaks() -> dict:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": float(d["hbm_gbs"]), "source": "measured (MEASURED_PEAKS.json)"}
+    return {"hbm_gbs": 6650.0, "source": "fallback (B200_PROFILING.md)"}
+
+
+def traffic_from_profile(kernel_key: str):
+    """dram read+write bytes per launch of the dominant kernel from the committed ncu --set full
+    summary (profiles/ncu_traffic.json), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        d = json.load(open(p))
+        return d.get(kernel_key)
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------------------------------------
+# CPU oracle leg (cpu_baseline and --impl reference)
+# ------------------------------------------------------------------------------------------------
+def oracle_band(cfg, P, row_start: int, nrows: int, host_rows=None, threads=None):
+    """Time the oracle (O1, all host cores) on rows [row_start, row_start+nrows) x all columns."""
+    import numpy as np
+
+    import oracle
+    from synth.dem import fill_host
+    threads = threads or os.cpu_count() or 1
+    if host_rows is None:
+        host_rows = fill_host(cfg.dem, cfg.cols, row_start, 0, nrows, cfg.cols, nthreads=threads)
+    bins = oracle.make_bins(cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata, oor_drop=cfg.oor_drop)
+    t0 = time.perf_counter()
+    H = oracle.o1(host_rows, cfg.gt, P, bins, row0=row_start, nthreads=threads)
+    dt = time.perf_counter() - t0
+    return dt, int(np.asarray(H).sum()), threads
+
+
+def calibrated_band(cfg, P, budget_s: float, row_mid: int | None = None, host=None, raster_dev=None):
+    """Pick a band of rows centred on row_mid whose oracle time is ~budget_s: probe bands of
+    doubling height until one takes >= budget_s / 8, then scale linearly."""
+    row_mid = cfg.rows // 2 if row_mid is None else row_mid
+    n = 64
+    while True:
+        n = min(n, cfg.rows)
+        start = max(0, min(cfg.rows - n, row_mid - n // 2))
+        if host is not None:
+            band = host[start:start + n, :cfg.cols]
+        elif raster_dev is not None:
+            band = raster_dev[start:start + n, :cfg.cols].cpu().numpy()
+        else:
+            band = None
+        dt, _, _ = oracle_band(cfg, P, start, n, host_rows=band)
+        if dt >= budget_s / 8 or n >= cfg.rows:
+            break
+        n *= 2
+    n = int(max(1, min(cfg.rows, n * budget_s / max(dt, 1e-6))))
+    start = max(0, min(cfg.rows - n, row_mid - n // 2))
+    return start, n
+
+
+def run_reference(args, cfg):
+    """Reference arm: the CPU oracle as it stands, on our config/metric, bounded sample per step."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    P = cfg.polygons()
+    budget = max(2.0, min(10.0, 150.0 / max(1, args.steps + args.warmup)))
+    start, n = calibrated_band(cfg, P, budget)
+    from synth.dem import fill_host
+    host = fill_host(cfg.dem, cfg.cols, start, 0, n, cfg.cols)
+    for _ in range(args.warmup):
+        oracle_band(cfg, P, start, n, host_rows=host)
+    times = []
+    threads = os.cpu_count() or 1
+    for _ in range(args.steps):
+        dt, _, threads = oracle_band(cfg, P, start, n, host_rows=host)
+        times.append(dt)
+    ms = 1000.0 * sum(times) / len(times)
+    cells = n * cfg.cols
+    value = cells / (ms / 1000.0)
+    sample = (f"rows [{start},{start + n}) x all {cfg.cols} cols of {cfg.name} ({cells} cells, "
+              f"{P.n_poly} polygons), oracle O1 (row-hoisted Franklin test), {threads} threads")
+    line = {"impl": "reference", "metric": "raster cells/s (zonal histogram, end-to-end)", "value": value,
+            "unit": "cells/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
+            "data": "synthetic", "config": cfg.describe(),
+            "cpu_baseline": {"value": value, "unit": "cells/s", "cores": threads, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "cells/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="conus")
+    ap.add_argument("--tile", type=int, default=None)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--verbose", action="store_true")
+    args = ap.parse_args()
+
+    from synth.configs import CONFIGS
+    cfg = CONFIGS[args.config]
+    if args.tile:
+        from dataclasses import replace
+        cfg = replace(cfg, tile=args.tile)
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangw14_b200 import zh
+    from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms, shard_rows
+    from synth.dem import fill_device
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    def log(*a):
+        if args.verbose and rank == 0:
+            print(*a, file=sys.stderr, flush=True)
+
+    t_setup = time.perf_counter()
+    P = cfg.polygons()
+    log(f"polygons: {P.n_poly} polys {P.n_vert} vertices ({time.perf_counter() - t_setup:.1f}s)")
+    T = cfg.tile
+    r0, r1 = shard_rows(cfg.rows, T, world, rank)
+    nrows = r1 - r0
+    pitch = (cfg.cols + 7) // 8 * 8
+    stream = torch.cuda.current_stream()
+    raster = torch.empty((max(nrows, 1), pitch), dtype=torch.int16, device="cuda")
+    fill_device(cfg.dem, cfg.cols, raster.data_ptr(), r0, 0, nrows, cfg.cols, pitch, stream.cuda_stream)
+    torch.cuda.synchronize()
+    log(f"raster shard rows [{r0},{r1}) generated ({time.perf_counter() - t_setup:.1f}s)")
+    raster_v = raster[:nrows]
+    out = torch.zeros((P.n_poly, cfg.nbins), dtype=torch.int64, device="cuda")
+    z = zh.ZonalHistogram(raster_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
+                          oor_drop=cfg.oor_drop, tile=T, rows=cfg.rows, cols=cfg.cols, row0=r0, stream=stream)
+    z.set_output(out)
+
+    steps_ev = []
+
+    def one_step(record=False):
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(5)] if record else None
+        if record:
+            evs[0].record(stream)
+        z.zh_pair_tiles()
+        if record:
+            evs[1].record(stream)
+        z.zh_tile_hist()
+        if record:
+            evs[2].record(stream)
+        z.zh_aggregate()
+        if record:
+            evs[3].record(stream)
+        z.zh_pip_update()
+        if record:
+            evs[4].record(stream)
+            steps_ev.append(evs)
+        if world > 1:
+            reduce_histograms(out)
+
+    clk = ClockSampler(local).__enter__()
+    time.sleep(0.5)  # nvidia-smi needs a moment before its first sample
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+    st = z.stats()
+    log(f"stats {st}")
+
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = z.launch_count()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        one_step(record=True)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clk.__exit__(None, None, None)
+    if world > 1:
+        dist.barrier()
+    launches = z.launch_count() - launches0
+    ms_local = e0.elapsed_time(e1) / args.steps
+    ms_t = torch.tensor([ms_local], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms = float(ms_t.item())
+    value = cfg.cells / (ms / 1000.0)
+
+    # per-step device times (averaged over the timed steps), rank-local
+    step_ms = [0.0] * 4
+    for evs in steps_ev:
+        for i in range(4):
+            step_ms[i] += evs[i].elapsed_time(evs[i + 1]) / len(steps_ev)
+    names = ["step2_pair_tiles", "step1_tile_hist", "step3_aggregate", "step4_pip_update"]
+    cells_local = nrows * cfg.cols
+    B_pad = (cfg.nbins + 3) // 4 * 4
+    alg_bytes = {
+        "step1_tile_hist": 2.0 * cells_local + 4.0 * B_pad * st["n_tiles"],
+        "step3_aggregate": 4.0 * cfg.nbins * st["n_inside"],
+        "step4_pip_update": 2.0 * st["n_isect"] * T * T,
+    }
+    peaks = measured_peaks()
+    dom = max(alg_bytes, key=lambda k: step_ms[names.index(k)])
+    dom_ms = step_ms[names.index(dom)]
+    achieved = alg_bytes[dom] / (dom_ms / 1000.0) / 1e9
+    kernel_name = {"step1_tile_hist": "k_tile_hist", "step3_aggregate": "k_aggregate", "step4_pip_update": "k_pip"}[dom]
+    roofline = {"bound": "hbm", "kernel": kernel_name, "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic_from_profile(kernel_name),
+                "peak_source": peaks["source"], "alg_bytes_per_launch": alg_bytes[dom],
+                "share_of_step": dom_ms / ms if ms > 0 else None}
+    steps_detail = {n: {"ms": step_ms[i]} for i, n in enumerate(names)}
+    for n, b in alg_bytes.items():
+        t = steps_detail[n]["ms"]
+        steps_detail[n]["alg_GBps"] = b / (t / 1000.0) / 1e9 if t > 0 else None
+    log(f"timed: {ms:.3f} ms/step, steps {steps_detail}")
+
+    # ---- end to end through the C ABI from host buffers
+    e2e = None
+    host = None
+    if not args.no_e2e:
+        e2e, host = run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log)
+    z.close()
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        start, n = calibrated_band(cfg, P, args.cpu_seconds, host=host, raster_dev=raster_v)
+        if host is not None:
+            band = host[start:start + n, :cfg.cols]
+        else:
+            band = raster_v[start:start + n, :cfg.cols].cpu().numpy()
+        dt, cnt, threads = oracle_band(cfg, P, start, n, host_rows=band)
+        cpu = {"value": n * cfg.cols / dt, "unit": "cells/s", "cores": threads, "kind": "oracle",
+               "sample": f"rows [{start},{start + n}) x all {cfg.cols} cols of {cfg.name} ({n * cfg.cols} cells, "
+                         f"{P.n_poly} polygons), oracle O1 on {threads} host threads, {dt:.1f} s"}
+
+    if rank == 0:
+        clocks = clk.summary()
+        line = {"metric": "raster cells/s (zonal histogram, end-to-end)", "value": value, "unit": "cells/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
+                "data": "synthetic (fractal int16 DEM + jagged Voronoi counties, seeded)",
+                "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert, parallelism=f"tile-row shards x{world}",
+                               l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA"),
+                "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
+                "clocks": clocks, "steps_detail": steps_detail, "pairs": {k: st[k] for k in
+                                                                         ("n_tiles", "n_candidates", "n_inside",
+                                                                          "n_isect", "n_band_entries", "n_edges")},
+                "setup_s": time.perf_counter() - t_setup}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log):
+    """E2E through the public API: host raster (pinned) + host polygons -> host histogram."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangw14_b200 import zh
+    from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms
+
+    # pinned host copy of this rank's strip (identical to the device one; D2H is not timed)
+    host = np.empty((max(nrows, 1), pitch), dtype=np.int16)
+    cudart = torch.cuda.cudart()
+    nbytes = host.nbytes
+    reg = cudart.cudaHostRegister(host.ctypes.data, nbytes, 0)
+    pinned = int(reg) == 0 if not isinstance(reg, tuple) else int(reg[0]) == 0
+    torch.from_numpy(host)[:nrows].copy_(raster_v)
+    torch.cuda.synchronize()
+    z.close()  # free the resident context's tile histograms before the e2e context allocates its own
+    res = np.empty((P.n_poly, cfg.nbins), dtype=np.uint64)
+    res_pin = torch.empty((P.n_poly, cfg.nbins), dtype=torch.int64, pin_memory=True)
+    host_v = host[:nrows]
+    times = []
+    for it in range(args.e2e_steps + 1):  # first iteration is a warm-up
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        z2 = zh.ZonalHistogram(host_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
+                               oor_drop=cfg.oor_drop, tile=cfg.tile, rows=cfg.rows, cols=cfg.cols, row0=r0,
+                               stream=stream)
+        if world > 1:
+            z2.set_output(out)
+            z2.zh_run(None)
+            reduce_histograms(out)
+            if rank == 0:
+                res_pin.copy_(out, non_blocking=True)
+            torch.cuda.synchronize()
+        else:
+            z2.zh_run(res)
+        dt = time.perf_counter() - t0
+        z2.close()
+        t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        if it > 0:
+            times.append(float(t.item()))
+    if pinned:
+        cudart.cudaHostUnregister(host.ctypes.data)
+    host = host[:nrows, :cfg.cols]
+    sec = sum(times) / len(times)
+    poly_bytes = P.x.nbytes + P.y.nbytes + P.poly_ring_off.nbytes // 2 + P.ring_vert_off.nbytes // 2
+    h2d = nrows * pitch * 2 + poly_bytes
+    if world > 1:
+        h2d_total = torch.tensor([h2d], dtype=torch.int64, device="cuda")
+        dist.all_reduce(h2d_total)
+        h2d = int(h2d_total.item())
+    d2h = P.n_poly * cfg.nbins * 8
+    log(f"e2e {sec:.3f} s/step (pinned={pinned})")
+    return {"value": cfg.cells / sec, "unit": "cells/s", "seconds_per_step": sec, "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": d2h, "host_raster_pinned": bool(pinned), "steps": len(times),
+            "includes": "zh_create (polygon H2D, allocation) + raster H2D + steps 2,1,3,4 + result D2H + zh_destroy"}, host
+
+
+if __name__ == "__main__":
+    sys.exit(main())
