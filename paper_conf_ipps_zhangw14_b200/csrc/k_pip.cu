@@ -17,9 +17,10 @@
 //     O(#(edge,row) crossings + cells) instead of O(cells x edges);
 //   * edges entirely left / right of the tile's centres (with half a cell of margin, far above
 //     the intercept's rounding) skip the division;
-//   * the cells are then streamed exactly like step 1 (16-byte vectors, inside-mask & nodata /
-//     bin mapping, run merging) into a CTA-private shared histogram, flushed once per pair with
-//     one global atomic per non-zero bin (no race).
+//   * the cells are then streamed exactly like step 1 (16-byte vectors, packed 16x2 bin mapping,
+//     one branch-free shared atomic per cell; vectors with no inside cell are not even loaded)
+//     into a CTA-private shared histogram, flushed once per pair with one global atomic per
+//     non-zero bin (no race).
 #include "zh_ctx.h"
 
 namespace zh {
@@ -36,6 +37,7 @@ struct PipP {
   const Edge* edges;
   const int2* erows;
   void* out;
+  FastBins fb;
   int B_pad;
   int wpr;  // bitmap words per row = T/32 + 1
   int rc;   // rows per chunk
@@ -52,11 +54,12 @@ __device__ __forceinline__ uint32_t bits8(const uint32_t* __restrict__ row, int 
   return (row[0] << (-lc0)) & 0xFFu;
 }
 
-template <bool kW1, bool kU64>
+template <int kMode, bool kU64>  // kMode as in k_tile_hist: 0/1 generic (w1 / w>1), 2 + kForm packed
 __global__ void __launch_bounds__(256) k_pip(PipP p) {
   extern __shared__ __align__(16) uint32_t sh[];
+  const int HW = hist_words(p.bp.nbins);
   uint32_t* hist = sh;
-  uint32_t* bm = sh + p.B_pad;
+  uint32_t* bm = sh + HW;
   const RasterP& rp = p.rp;
   const Geo& g = p.g;
 
@@ -77,12 +80,15 @@ __global__ void __launch_bounds__(256) k_pip(PipP p) {
   const double xlo_t = fmin(xa_t, xb_t), xhi_t = fmax(xa_t, xb_t);
   const double half = 0.5 * fabs(g.gt1);
 
-  for (int i = threadIdx.x * 4; i < p.B_pad; i += blockDim.x * 4)
+  for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
     *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
+  const uint32_t dummy = (uint32_t)hist_dummy(p.bp.nbins) + (threadIdx.x & 31);
+  const uint32_t dum2 = dummy * 0x10001u;
 
   const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
   const int nk = (int)(k1 - k0);
   const int64_t pitch = rp.pitch;
+  const FastBins fb = p.fb;
 
   for (int cr = 0; cr < h; cr += p.rc) {
     const int ch = min(p.rc, h - cr);
@@ -132,18 +138,36 @@ __global__ void __launch_bounds__(256) k_pip(PipP p) {
       }
     }
     __syncthreads();
-    // ---- cells: stream the chunk's rows, count inside cells
+    // ---- cells: stream the chunk's rows, count inside cells (fully-outside vectors are not read)
     const int16_t* base = rp.data + (rlo - rp.row0) * pitch + k0 * 8;
-    for (int idx = threadIdx.x; idx < ch * nk; idx += blockDim.x) {
-      const int lr = idx / nk, kk = idx - lr * nk;
-      const int64_t cs = (k0 + kk) * 8;
-      uint32_t valid = 0xFFu;
-      if (cs < c0) valid &= (0xFFu << (int)(c0 - cs)) & 0xFFu;
-      if (cs + 8 > c0 + w) valid &= 0xFFu >> (int)(cs + 8 - (c0 + w));
-      valid &= bits8(bm + lr * p.wpr, p.wpr, (int)(cs - c0));
-      if (!valid) continue;
-      const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
-      count8<kW1>(hist, q, valid, p.bp);
+    if (nk <= (int)blockDim.x) {
+      const int rpi = blockDim.x / nk;
+      const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
+      if (rs < rpi) {
+        const int64_t cs = (k0 + kk) * 8;
+        const uint32_t cskip = cols_skip8(cs, c0, w);
+        const int lc0 = (int)(cs - c0);
+        const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
+        const int64_t step = (int64_t)rpi * pitch;
+        for (int lr = rs; lr < ch; lr += rpi, ptr += step) {
+          const uint32_t skip = cskip | (~bits8(bm + lr * p.wpr, p.wpr, lc0) & 0xFFu);
+          if (skip == 0xFFu) continue;
+          const uint4 q = ld_stream16(ptr);
+          if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q, skip, fb, dum2);
+          else count8_generic<kMode == 0>(hist, q, skip, p.bp, dummy);
+        }
+      }
+    } else {
+      for (int lr = 0; lr < ch; ++lr) {
+        for (int kk = threadIdx.x; kk < nk; kk += blockDim.x) {
+          const int64_t cs = (k0 + kk) * 8;
+          const uint32_t skip = cols_skip8(cs, c0, w) | (~bits8(bm + lr * p.wpr, p.wpr, (int)(cs - c0)) & 0xFFu);
+          if (skip == 0xFFu) continue;
+          const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
+          if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q, skip, fb, dum2);
+          else count8_generic<kMode == 0>(hist, q, skip, p.bp, dummy);
+        }
+      }
     }
     __syncthreads();
   }
@@ -151,7 +175,7 @@ __global__ void __launch_bounds__(256) k_pip(PipP p) {
   const int nbins = p.bp.nbins;
   const int64_t orow = (int64_t)k * nbins;
   for (int b = threadIdx.x; b < nbins; b += blockDim.x) {
-    const uint32_t v = hist[b];
+    const uint32_t v = hist[kOff + b];
     if (v) {
       if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(p.out) + orow + b, (unsigned long long)v);
       else atomicAdd(reinterpret_cast<uint32_t*>(p.out) + orow + b, v);
@@ -174,16 +198,23 @@ cudaError_t launch_pip(Ctx& c) {
   p.erows = c.d_erows.as<int2>();
   p.out = c.d_out;
   p.B_pad = c.B_pad;
+  p.fb = make_fast_bins(c.bp);
   p.wpr = c.rp.T / 32 + 1;
   const int bm_budget_words = 8192;  // 32 KB of parity bitmap per CTA
   p.rc = bm_budget_words / p.wpr;
   if (p.rc < 1) p.rc = 1;
   if (p.rc > c.rp.T) p.rc = c.rp.T;
-  const size_t smem = (size_t)c.B_pad * 4 + (size_t)p.rc * p.wpr * 4;
+  const size_t smem = (size_t)hist_words(c.bp.nbins) * 4 + (size_t)p.rc * p.wpr * 4;
   const int threads = 256;
   void (*k)(PipP);
-  if (c.bp.width == 1) k = c.out_u64 ? k_pip<true, true> : k_pip<true, false>;
-  else k = c.out_u64 ? k_pip<false, true> : k_pip<false, false>;
+  const int mode = fast_bins_ok(c.bp) ? (p.fb.bias ? 4 : (c.bp.use_nodata ? 3 : 2)) : (c.bp.width == 1 ? 0 : 1);
+  switch (mode) {
+    case 0: k = c.out_u64 ? k_pip<0, true> : k_pip<0, false>; break;
+    case 1: k = c.out_u64 ? k_pip<1, true> : k_pip<1, false>; break;
+    case 2: k = c.out_u64 ? k_pip<2, true> : k_pip<2, false>; break;
+    case 3: k = c.out_u64 ? k_pip<3, true> : k_pip<3, false>; break;
+    default: k = c.out_u64 ? k_pip<4, true> : k_pip<4, false>; break;
+  }
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k<<<(unsigned)c.n_isect, threads, smem, c.stream>>>(p);
   c.launches += 1;

@@ -4,19 +4,23 @@
 //
 // Paper design (prior art): one thread block per tile, 256 threads, a global-memory atomicAdd per
 // cell.  B200 design: one CTA per tile with the tile's histogram privatised in SHARED memory
-// (B_pad x 4 bytes, 20 KB at B = 5000), raster read as 16-byte streaming vectors (8 int16 cells,
-// ld.global.nc.L1::no_allocate), 4 independent 16-byte loads in flight per thread, runs of equal
-// bins inside each vector merged in registers before the shared atomic, and one coalesced 16-byte
-// store pass per tile (no global zeroing pass).  HBM-bound: 2 B/cell read + 4*B_pad/T^2 B/cell
-// written.
+// (20 KB at B = 5000); the raster is read as 16-byte streaming vectors (8 int16 cells,
+// ld.global.nc.L1::no_allocate), 4 independent vectors in flight per thread; bins are computed
+// two cells at a time with packed 16x2 min/max/add (VIMNMX.S16x2 / VIADD.16x2) and a zero-detect
+// for nodata; every cell then issues exactly one shared atomic with no predicate or branch —
+// cells that are not counted go to one of 32 per-lane dummy slots (zh_internal.cuh, HistLayout).
+// The histogram leaves with one coalesced 16-byte store pass per tile (no global zeroing pass).
+// HBM-bound: 2 B/cell read + 4*B_pad/T^2 B/cell written.
 #include "zh_ctx.h"
 
 namespace zh {
 
-template <bool kW1>
-__global__ void __launch_bounds__(512) k_tile_hist(RasterP rp, BinP bp, int B_pad,
+// kMode: 0 generic bins (width 1), 1 generic bins (width > 1), 2 + kForm: packed bins (fast_idx2)
+template <int kMode>
+__global__ void __launch_bounds__(512) k_tile_hist(RasterP rp, BinP bp, FastBins fb, int B_pad,
                                                    uint32_t* __restrict__ tile_hist) {
   extern __shared__ __align__(16) uint32_t sh[];
+  const int HW = hist_words(bp.nbins);
   const int tile = blockIdx.x;
   const int tr = tile / rp.TC, tc = tile - tr * rp.TC;
   const int64_t r0 = (int64_t)(rp.tr0 + tr) * rp.T;
@@ -24,9 +28,20 @@ __global__ void __launch_bounds__(512) k_tile_hist(RasterP rp, BinP bp, int B_pa
   const int64_t c0 = (int64_t)tc * rp.T;
   const int w = (int)min((int64_t)rp.T, rp.cols - c0);
 
-  for (int i = threadIdx.x * 4; i < B_pad; i += blockDim.x * 4)
+  for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
     *reinterpret_cast<uint4*>(&sh[i]) = make_uint4(0, 0, 0, 0);
   __syncthreads();
+
+  const uint32_t dummy = (uint32_t)hist_dummy(bp.nbins) + (threadIdx.x & 31);
+  const uint32_t dum2 = dummy * 0x10001u;
+  auto count = [&](const uint4& q, uint32_t skip) {
+    if (kMode >= 2) {
+      if (skip == 0) count8_fast<kMode - 2, false>(sh, q, 0, fb, dum2);
+      else count8_fast<kMode - 2, true>(sh, q, skip, fb, dum2);
+    } else {
+      count8_generic<kMode == 0>(sh, q, skip, bp, dummy);
+    }
+  };
 
   const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
   const int nk = (int)(k1 - k0);
@@ -37,53 +52,55 @@ __global__ void __launch_bounds__(512) k_tile_hist(RasterP rp, BinP bp, int B_pa
     const int rpi = blockDim.x / nk;  // rows per block iteration
     const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
     if (rs < rpi) {
-      const int64_t cs = (k0 + kk) * 8;
-      uint32_t valid = 0xFFu;
-      if (cs < c0) valid &= (0xFFu << (int)(c0 - cs)) & 0xFFu;
-      if (cs + 8 > c0 + w) valid &= 0xFFu >> (int)(cs + 8 - (c0 + w));
-      const int16_t* p = base + kk * 8;
+      const uint32_t skip = cols_skip8((k0 + kk) * 8, c0, w);
+      const int16_t* p = base + (int64_t)rs * pitch + kk * 8;
+      const int64_t step = (int64_t)rpi * pitch;
       int r = rs;
       for (; r + 3 * rpi < h; r += 4 * rpi) {
-        const uint4 q0 = ld_stream16(p + (int64_t)r * pitch);
-        const uint4 q1 = ld_stream16(p + (int64_t)(r + rpi) * pitch);
-        const uint4 q2 = ld_stream16(p + (int64_t)(r + 2 * rpi) * pitch);
-        const uint4 q3 = ld_stream16(p + (int64_t)(r + 3 * rpi) * pitch);
-        count8<kW1>(sh, q0, valid, bp);
-        count8<kW1>(sh, q1, valid, bp);
-        count8<kW1>(sh, q2, valid, bp);
-        count8<kW1>(sh, q3, valid, bp);
+        const uint4 q0 = ld_stream16(p);
+        const uint4 q1 = ld_stream16(p + step);
+        const uint4 q2 = ld_stream16(p + 2 * step);
+        const uint4 q3 = ld_stream16(p + 3 * step);
+        p += 4 * step;
+        count(q0, skip);
+        count(q1, skip);
+        count(q2, skip);
+        count(q3, skip);
       }
-      for (; r < h; r += rpi) count8<kW1>(sh, ld_stream16(p + (int64_t)r * pitch), valid, bp);
+      for (; r < h; r += rpi, p += step) count(ld_stream16(p), skip);
     }
   } else {
     for (int r = 0; r < h; ++r) {
-      for (int kk = threadIdx.x; kk < nk; kk += blockDim.x) {
-        const int64_t cs = (k0 + kk) * 8;
-        uint32_t valid = 0xFFu;
-        if (cs < c0) valid &= (0xFFu << (int)(c0 - cs)) & 0xFFu;
-        if (cs + 8 > c0 + w) valid &= 0xFFu >> (int)(cs + 8 - (c0 + w));
-        count8<kW1>(sh, ld_stream16(base + (int64_t)r * pitch + kk * 8), valid, bp);
-      }
+      for (int kk = threadIdx.x; kk < nk; kk += blockDim.x)
+        count(ld_stream16(base + (int64_t)r * pitch + kk * 8), cols_skip8((k0 + kk) * 8, c0, w));
     }
   }
   __syncthreads();
   uint32_t* dst = tile_hist + (int64_t)tile * B_pad;
   for (int i = threadIdx.x * 4; i < B_pad; i += blockDim.x * 4)
-    *reinterpret_cast<uint4*>(&dst[i]) = *reinterpret_cast<const uint4*>(&sh[i]);
+    *reinterpret_cast<uint4*>(&dst[i]) = *reinterpret_cast<const uint4*>(&sh[kOff + i]);
+}
+
+template <int kMode>
+static void launch_mode(Ctx& c, size_t smem, int threads) {
+  auto k = k_tile_hist<kMode>;
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<(unsigned)c.n_tiles, threads, smem, c.stream>>>(c.rp, c.bp, make_fast_bins(c.bp), c.B_pad,
+                                                      c.d_tile_hist.as<uint32_t>());
 }
 
 cudaError_t launch_tile_hist(Ctx& c) {
   if (c.n_tiles == 0) return cudaSuccess;
-  const size_t smem = (size_t)c.B_pad * 4;
+  const size_t smem = (size_t)hist_words(c.bp.nbins) * 4;
   const int threads = 512;
-  if (c.bp.width == 1) {
-    auto k = k_tile_hist<true>;
-    if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k<<<(unsigned)c.n_tiles, threads, smem, c.stream>>>(c.rp, c.bp, c.B_pad, c.d_tile_hist.as<uint32_t>());
+  if (fast_bins_ok(c.bp)) {
+    const FastBins f = make_fast_bins(c.bp);
+    if (f.bias) launch_mode<4>(c, smem, threads);
+    else if (c.bp.use_nodata) launch_mode<3>(c, smem, threads);
+    else launch_mode<2>(c, smem, threads);
   } else {
-    auto k = k_tile_hist<false>;
-    if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k<<<(unsigned)c.n_tiles, threads, smem, c.stream>>>(c.rp, c.bp, c.B_pad, c.d_tile_hist.as<uint32_t>());
+    if (c.bp.width == 1) launch_mode<0>(c, smem, threads);
+    else launch_mode<1>(c, smem, threads);
   }
   c.launches += 1;
   return cudaGetLastError();

@@ -92,26 +92,132 @@ __device__ __forceinline__ int cell_of(const uint4& q, int j) {
   return (int)(int16_t)(w >> ((j & 1) * 16));
 }
 
-// Count the valid cells (bit j of `valid`) of an 8-cell vector into a shared-memory histogram.
-// Runs of equal bins inside the vector are merged first (DEM neighbours are often equal, so this
-// removes same-address serialisation of the shared atomics).
+// ----------------------------------------------------------------------------------------------
+// Shared-memory histogram layout used by steps 1 and 4 (HistLayout):
+//   hist[kOff - 1]            "below range" trash (drop mode)
+//   hist[kOff + b]            bin b, b in [0, nbins)          (16-byte aligned: kOff = 4)
+//   hist[kOff + nbins]        "above range" trash (drop mode)
+//   hist[dum + lane]          32 per-lane dummy slots for cells that are not counted (nodata,
+//                             outside the tile / polygon): every cell issues exactly one shared
+//                             atomic, with no predicate and no branch, and the not-counted
+//                             ones never collide across lanes.
+// ----------------------------------------------------------------------------------------------
+constexpr int kOff = 4;
+
+__host__ __device__ __forceinline__ int hist_dummy(int nbins) { return (kOff + nbins + 1 + 3) & ~3; }
+__host__ __device__ __forceinline__ int hist_words(int nbins) { return hist_dummy(nbins) + 32; }
+
+// Packed 16x2 bin mapping (width == 1, lo in int16, nbins <= 16000; see fast_bins_ok).
+// Two formulations, both ending with idx in [kOff-1, kOff+nbins] for counted cells and a value
+// >= the dummy base for cells that are not counted:
+//  kBias (use_nodata and nodata < L, e.g. SRTM voids = -32768 below every bin):
+//     a = min_s16(v, H); b = a - (nodata+1) (mod 2^16)   -> nodata becomes 0xFFFF, the rest keep order
+//     c = max_u16(b, L - nodata - 1); idx = c - (C - nodata - 1)
+//     (nodata stays far above the dummy base; 4 ALU ops per two cells, no compare)
+//  plain (no nodata, or nodata inside the range):
+//     c = clamp_s16(v, L, H); idx = c - C; nodata halves -> 0xFFFF by a zero-detect of v ^ nodata
+// clamp mode: L = lo, H = lo+nbins-1 (capped at 32767)   drop mode: L = lo-1, H = lo+nbins (trash)
+// C = lo - kOff.
+struct FastBins {
+  uint32_t L2, H2, C2, nod2;   // plain
+  uint32_t Hb2, Nb2, Lb2, Cb2;  // biased
+  uint32_t use_nodata, bias;
+};
+
+__host__ __device__ inline bool fast_bins_ok(const BinP& b) {
+  return b.width == 1 && b.lo >= -32768 && b.lo <= 32767 && b.nbins <= 16000;
+}
+
+__host__ __device__ inline FastBins make_fast_bins(const BinP& b) {
+  FastBins f;
+  const int top = b.lo + b.nbins - 1;  // last value with a bin of its own
+  int L = b.lo, H = top < 32767 ? top : 32767;
+  if (b.drop) {
+    if (b.lo > -32768) L = b.lo - 1;  // below-range trash; nothing is below -32768
+    if (top < 32767) H = top + 1;     // above-range trash; nothing is above 32767
+  }
+  const int C = b.lo - kOff;
+  auto pk = [](int v) { return (uint32_t)(uint16_t)v * 0x10001u; };
+  f.L2 = pk(L);
+  f.H2 = pk(H);
+  f.C2 = pk(C);
+  f.nod2 = pk(b.nodata);
+  f.use_nodata = b.use_nodata ? 1u : 0u;
+  // biased form: valid when nodata < L and the nodata index stays above the dummy slots
+  const int N1 = b.nodata + 1;
+  f.Hb2 = pk(H);
+  f.Nb2 = pk(N1);
+  f.Lb2 = pk(L - N1);
+  f.Cb2 = pk(C - N1);
+  const int nod_idx = 0xFFFF - ((C - N1) & 0xFFFF);  // where a nodata cell lands
+  f.bias = (b.use_nodata && b.nodata < L && nod_idx >= hist_dummy(b.nbins) + 32) ? 1u : 0u;
+  return f;
+}
+
+template <int kForm>  // 0 plain, 1 plain + nodata zero-detect, 2 biased (nodata below range)
+__device__ __forceinline__ uint32_t fast_idx2(uint32_t w, const FastBins& f) {
+  if (kForm == 2) {
+    uint32_t a = __vmins2(w, f.Hb2);
+    a = __vsub2(a, f.Nb2);
+    a = __vmaxu2(a, f.Lb2);
+    return __vsub2(a, f.Cb2);
+  }
+  uint32_t c = __vmaxs2(w, f.L2);
+  c = __vmins2(c, f.H2);
+  c = __vsub2(c, f.C2);
+  if (kForm == 1) {
+    const uint32_t x = w ^ f.nod2;                 // zero halves where v == nodata
+    const uint32_t z = __vsub2(x, 0x00010001u) & ~x & 0x80008000u;
+    c |= __byte_perm(z, 0, 0xBB99);                // 0xFFFF in those halves
+  }
+  return c;
+}
+
+// Byte j of the result pair (lo: cells 0-3, hi: cells 4-7) is 0xFF when bit j of m is set.
+__device__ __forceinline__ void spread_bits8(uint32_t m, uint32_t& lo, uint32_t& hi) {
+  lo = (((m & 0xFu) * 0x00204081u) & 0x01010101u) * 0xFFu;
+  hi = ((((m >> 4) & 0xFu) * 0x00204081u) & 0x01010101u) * 0xFFu;
+}
+
+// Count 8 cells (one 16-byte vector) into the shared histogram.  `skip` has bit j set for cells
+// that must not be counted (outside the tile / not inside the polygon).  `dum2` = (dummy slot
+// of this lane) in both halves.  Indices are < 2^14, so idx*4 of both halves is one 32-bit
+// shift of the packed pair.
+template <int kForm, bool kMask>
+__device__ __forceinline__ void count8_fast(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                            const FastBins& f, uint32_t dum2) {
+  uint32_t sl = 0, sh = 0;
+  if (kMask) spread_bits8(skip, sl, sh);
+  const uint32_t ws[4] = {q.x, q.y, q.z, q.w};
+  char* hb = reinterpret_cast<char*>(hist);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    uint32_t x = fast_idx2<kForm>(ws[i], f);
+    if (kMask) x |= __byte_perm(sl, sh, (uint32_t)((2 * i) | (2 * i) << 4 | (2 * i + 1) << 8 | (2 * i + 1) << 12));
+    x = __vminu2(x, dum2) << 2;  // byte offsets of both cells
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);
+  }
+}
+
+// Generic path (any width / lo / nbins): same layout, scalar mapping, per-cell atomics.
 template <bool kW1>
-__device__ __forceinline__ void count8(uint32_t* __restrict__ hist, const uint4& q, uint32_t valid,
-                                       const BinP& bp) {
-  int prev = -1;
-  uint32_t run = 0;
+__device__ __forceinline__ void count8_generic(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                               const BinP& bp, uint32_t dummy) {
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
-    int b = ((valid >> j) & 1u) ? bin_of<kW1>(cell_of(q, j), bp) : -1;
-    if (b == prev) {
-      ++run;
-    } else {
-      if (prev >= 0) atomicAdd(&hist[prev], run);
-      prev = b;
-      run = 1;
-    }
+    int b = ((skip >> j) & 1u) ? -1 : bin_of<kW1>(cell_of(q, j), bp);
+    atomicAdd(&hist[b >= 0 ? kOff + b : (int)dummy], 1u);
   }
-  if (prev >= 0) atomicAdd(&hist[prev], run);
+}
+
+// Validity of the 8 cells starting at column cs within the tile columns [c0, c0 + w): bit j set
+// when column cs + j is OUTSIDE (to be skipped).
+__device__ __forceinline__ uint32_t cols_skip8(int64_t cs, int64_t c0, int w) {
+  uint32_t valid = 0xFFu;
+  if (cs < c0) valid &= (0xFFu << (int)(c0 - cs)) & 0xFFu;
+  if (cs + 8 > c0 + w) valid &= 0xFFu >> (int)(cs + 8 - (c0 + w));
+  return ~valid & 0xFFu;
 }
 
 // ----------------------------------------------------------------------------------------------
