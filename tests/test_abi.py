@@ -43,21 +43,34 @@ def test_library_is_sm100a_sass():
     assert "sm_100a" in out
 
 
+def _sass_functions(lib):
+    out = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True, check=True).stdout
+    funcs, cur = {}, None
+    for line in out.splitlines():
+        m = re.match(r"\s+Function : (\S+)", line)
+        if m:
+            cur = m.group(1)
+            funcs[cur] = []
+        elif cur is not None:
+            funcs[cur].append(line)
+    return funcs
+
+
 def test_pip_predicate_has_no_contracted_fma():
-    """The intercept / centre expressions must be separate DMUL/DADD (R7).  DFMA may only appear
-    inside the IEEE division routine; check that every DFMA sits in a division sequence by
-    verifying the kernel's DFMA count equals that of a kernel with only the divisions."""
+    """The intercept / centre expressions are written with __dadd_rn/__dsub_rn/__dmul_rn/__ddiv_rn
+    (R7), which nvcc never contracts.  Weak SASS check on every kernel evaluating the predicate:
+    DMUL and DADD are present, and DFMA appears only as part of division sequences (each IEEE
+    double division is an MUFU.RCP64H followed by a handful of DFMAs)."""
     from paper_conf_ipps_zhangw14_b200 import _build
-    lib = _build.build()
-    sass = subprocess.run(["cuobjdump", "-sass", "-fun", "_ZN2zh5k_pipILb1ELb1EEEvNS_4PipPE", lib],
-                          capture_output=True, text=True, check=True).stdout
-    assert "DMUL" in sass and "DADD" in sass
-    # the division routine's DFMAs follow an MUFU.RCP64H; no DFMA may consume the centre/intercept
-    # operands directly — weak check: DFMA count is bounded by the number of reciprocal sequences
-    n_dfma = sass.count("DFMA")
-    n_rcp = sass.count("MUFU.RCP64H")
-    assert n_rcp >= 1
-    assert n_dfma <= 8 * n_rcp + 8
+    funcs = _sass_functions(_build.build())
+    names = [n for n in funcs if any(k in n for k in ("k_pip", "k_classify", "k_edges"))]
+    assert names
+    for n in names:
+        sass = "\n".join(funcs[n])
+        assert "DMUL" in sass and "DADD" in sass, n
+        n_rcp = sass.count("MUFU.RCP64H")
+        assert n_rcp >= 1, n
+        assert sass.count("DFMA") <= 10 * n_rcp, n
 
 
 def _mk(lib_zh, **over):

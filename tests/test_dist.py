@@ -1,0 +1,84 @@
+"""Multi-GPU host logic on CPU: tile-row sharding and the histogram reduction (gloo, world 2).
+
+The per-rank compute here is the oracle on the rank's strip (the GPU shard path is covered by
+tests/test_gpu_parity.py::test_tile_row_shards_sum_to_whole); what is tested is that the strips
+partition the raster into whole tile rows and that the all-reduce of the partial histograms
+(int64 view of uint64 counts) reproduces the single-process result bit for bit.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms, shard_rows
+
+
+@pytest.mark.parametrize("rows,tile,world", [(1024, 128, 2), (1000, 96, 3), (93600, 256, 8), (5, 7, 4),
+                                             (0, 16, 2), (256, 256, 8)])
+def test_shard_rows_partition_whole_tile_rows(rows, tile, world):
+    spans = [shard_rows(rows, tile, world, r) for r in range(world)]
+    assert spans[0][0] == 0 and spans[-1][1] == rows
+    for (a0, a1), (b0, b1) in zip(spans, spans[1:]):
+        assert a1 == b0
+    for r0, r1 in spans:
+        assert r0 <= r1 and r0 % tile == 0 or r0 == rows
+
+
+def test_shard_rows_rejects_bad_args():
+    with pytest.raises(ValueError):
+        shard_rows(10, 0, 2, 0)
+    with pytest.raises(ValueError):
+        shard_rows(10, 4, 2, 2)
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from synth.configs import TINY as cfg
+        from synth.dem import fill_host
+        P = cfg.polygons()
+        r0, r1 = shard_rows(cfg.rows, cfg.tile, world, rank)
+        R = fill_host(cfg.dem, cfg.cols, r0, 0, r1 - r0, cfg.cols, nthreads=2)
+        H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata), row0=r0, nthreads=2)
+        t = torch.from_numpy(H.view(np.int64).copy())
+        reduce_histograms(t)
+        q.put((rank, t.numpy().view(np.uint64).copy()))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_reduce_equals_single_process():
+    import oracle
+    from synth.configs import TINY as cfg
+    from synth.dem import fill_host
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    P = cfg.polygons()
+    R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata))
+    for r in range(world):
+        assert (res[r] == H).all()
