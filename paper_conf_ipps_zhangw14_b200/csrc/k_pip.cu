@@ -149,7 +149,24 @@ __global__ void __launch_bounds__(256) k_pip(PipP p) {
         const int lc0 = (int)(cs - c0);
         const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
         const int64_t step = (int64_t)rpi * pitch;
-        for (int lr = rs; lr < ch; lr += rpi, ptr += step) {
+        int lr = rs;
+        // two rows per iteration: both skip masks first, then both loads in flight
+        for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
+          const uint32_t s0 = cskip | (~bits8(bm + lr * p.wpr, p.wpr, lc0) & 0xFFu);
+          const uint32_t s1 = cskip | (~bits8(bm + (lr + rpi) * p.wpr, p.wpr, lc0) & 0xFFu);
+          uint4 q0 = make_uint4(0, 0, 0, 0), q1 = make_uint4(0, 0, 0, 0);
+          if (s0 != 0xFFu) q0 = ld_stream16(ptr);
+          if (s1 != 0xFFu) q1 = ld_stream16(ptr + step);
+          if (s0 != 0xFFu) {
+            if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q0, s0, fb, dum2);
+            else count8_generic<kMode == 0>(hist, q0, s0, p.bp, dummy);
+          }
+          if (s1 != 0xFFu) {
+            if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q1, s1, fb, dum2);
+            else count8_generic<kMode == 0>(hist, q1, s1, p.bp, dummy);
+          }
+        }
+        for (; lr < ch; lr += rpi, ptr += step) {
           const uint32_t skip = cskip | (~bits8(bm + lr * p.wpr, p.wpr, lc0) & 0xFFu);
           if (skip == 0xFFu) continue;
           const uint4 q = ld_stream16(ptr);

@@ -17,7 +17,7 @@ namespace zh {
 
 // kMode: 0 generic bins (width 1), 1 generic bins (width > 1), 2 + kForm: packed bins (fast_idx2)
 template <int kMode>
-__global__ void __launch_bounds__(512) k_tile_hist(RasterP rp, BinP bp, FastBins fb, int B_pad,
+__global__ void __launch_bounds__(512, 3) k_tile_hist(RasterP rp, BinP bp, FastBins fb, int B_pad,
                                                    uint32_t* __restrict__ tile_hist) {
   extern __shared__ __align__(16) uint32_t sh[];
   const int HW = hist_words(bp.nbins);

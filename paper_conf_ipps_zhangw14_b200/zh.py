@@ -16,7 +16,8 @@ import numpy as np
 
 from . import _build
 
-_LIB_PATH = _build.LIB
+# ZH_LIBZH: load another build of libzh (A/B experiments); default is the in-tree build.
+_LIB_PATH = os.environ.get("ZH_LIBZH", _build.LIB)
 
 ZH_OK, ZH_ERR_INVALID_ARG, ZH_ERR_UNSUPPORTED, ZH_ERR_OOM, ZH_ERR_CUDA, ZH_ERR_OVERFLOW, ZH_ERR_STATE = range(7)
 _STATUS = {0: "ZH_OK", 1: "ZH_ERR_INVALID_ARG", 2: "ZH_ERR_UNSUPPORTED", 3: "ZH_ERR_OOM", 4: "ZH_ERR_CUDA",
