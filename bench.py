@@ -2,7 +2,8 @@
 """bench.py — zonal histogramming throughput on B200 (raster cells/s, end-to-end), driver contract.
 
 A "step" is one pass of the whole hot path: zh_pair_tiles (step 2, incl.
-zeroing the output), zh_tile_hist (step 1), zh_aggregate (step 3), zh_pip_update (step 4) over
+zeroing the output) then zh_fused_update (steps 1 + 3 + 4 fused tile by tile, SURVEY.md §8f-1;
+`--path four_step` runs zh_tile_hist, zh_aggregate, zh_pip_update instead — both are timed) over
 the CONUS-scale synthetic raster (93,600 x 216,000 int16 = 20.2 G cells, 40.4 GB resident in HBM)
 and ~3,100 jagged county polygons; with N > 1 GPUs each rank holds a strip of whole tile rows
 and the step ends with an NCCL all-reduce of the [n_poly, 5000] uint64 histograms.
@@ -201,6 +202,9 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--verbose", action="store_true")
+    ap.add_argument("--path", default="fused", choices=["fused", "four_step"],
+                    help="fused: step 2 + zh_fused_update (steps 1+3+4 fused, SURVEY §8f-1); four_step: 2,1,3,4")
+    ap.add_argument("--no-other", action="store_true", help="skip timing the other path")
     args = ap.parse_args()
 
     from synth.configs import CONFIGS
@@ -245,28 +249,25 @@ def main():
     raster_v = raster[:nrows]
     out = torch.zeros((P.n_poly, cfg.nbins), dtype=torch.int64, device="cuda")
     z = zh.ZonalHistogram(raster_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
-                          oor_drop=cfg.oor_drop, tile=T, rows=cfg.rows, cols=cfg.cols, row0=r0, stream=stream)
+                          oor_drop=cfg.oor_drop, tile=T, rows=cfg.rows, cols=cfg.cols, row0=r0, stream=stream,
+                          fused=(args.path == "fused"))
     z.set_output(out)
 
-    steps_ev = []
+    path = args.path
+    z.set_timing(True)
+    lib_ms = []  # per timed step: the library's own event timings (steps, fused inner kernels)
 
-    def one_step(record=False):
-        evs = [torch.cuda.Event(enable_timing=True) for _ in range(5)] if record else None
-        if record:
-            evs[0].record(stream)
+    def one_step(record=False, mode=None):
+        mode = mode or path
         z.zh_pair_tiles()
+        if mode == "fused":
+            z.zh_fused_update()
+        else:
+            z.zh_tile_hist()
+            z.zh_aggregate()
+            z.zh_pip_update()
         if record:
-            evs[1].record(stream)
-        z.zh_tile_hist()
-        if record:
-            evs[2].record(stream)
-        z.zh_aggregate()
-        if record:
-            evs[3].record(stream)
-        z.zh_pip_update()
-        if record:
-            evs[4].record(stream)
-            steps_ev.append(evs)
+            lib_ms.append(z.step_ms())  # syncs after the step's last kernel
         if world > 1:
             reduce_histograms(out)
 
@@ -299,34 +300,68 @@ def main():
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms = float(ms_t.item())
     value = cfg.cells / (ms / 1000.0)
+    st = z.stats()
 
-    # per-step device times (averaged over the timed steps), rank-local
-    step_ms = [0.0] * 4
-    for evs in steps_ev:
-        for i in range(4):
-            step_ms[i] += evs[i].elapsed_time(evs[i + 1]) / len(steps_ev)
-    names = ["step2_pair_tiles", "step1_tile_hist", "step3_aggregate", "step4_pip_update"]
+    def avg(rows, key):
+        v = [r[key] for r in rows if r[key] >= 0]
+        return sum(v) / len(v) if v else None
+
+    peaks = measured_peaks()
     cells_local = nrows * cfg.cols
     B_pad = (cfg.nbins + 3) // 4 * 4
-    alg_bytes = {
-        "step1_tile_hist": 2.0 * cells_local + 4.0 * B_pad * st["n_tiles"],
-        "step3_aggregate": 4.0 * cfg.nbins * st["n_inside"],
-        "step4_pip_update": 2.0 * st["n_isect"] * T * T,
-    }
-    peaks = measured_peaks()
-    dom = max(alg_bytes, key=lambda k: step_ms[names.index(k)])
-    dom_ms = step_ms[names.index(dom)]
-    achieved = alg_bytes[dom] / (dom_ms / 1000.0) / 1e9
-    kernel_name = {"step1_tile_hist": "k_tile_hist", "step3_aggregate": "k_aggregate", "step4_pip_update": "k_pip"}[dom]
-    roofline = {"bound": "hbm", "kernel": kernel_name, "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic_from_profile(kernel_name),
-                "peak_source": peaks["source"], "alg_bytes_per_launch": alg_bytes[dom],
+    # algorithmic bytes per launch
+    kern = {}
+    if path == "fused":
+        kern["k_fused_pure"] = (avg(lib_ms, "fused_pure_kernel"), 2.0 * st["n_pure_cells"])
+        kern["k_pip"] = (avg(lib_ms, "fused_pip_kernel"), 2.0 * st["n_pip_cells"])
+        steps_detail = {"step2_pair_tiles": {"ms": avg(lib_ms, "step2_pair_tiles")},
+                        "fused_update(steps1+3+4)": {"ms": avg(lib_ms, "fused_update")}}
+    else:
+        kern["k_tile_hist"] = (avg(lib_ms, "step1_tile_hist"), 2.0 * cells_local + 4.0 * B_pad * st["n_tiles"])
+        kern["k_aggregate"] = (avg(lib_ms, "step3_aggregate"), 4.0 * cfg.nbins * st["n_inside"])
+        kern["k_pip"] = (avg(lib_ms, "step4_pip_update"), 2.0 * st["n_isect"] * T * T)
+        steps_detail = {"step2_pair_tiles": {"ms": avg(lib_ms, "step2_pair_tiles")}}
+    for name, (t, b) in kern.items():
+        steps_detail[name] = {"ms": t, "alg_bytes": b, "alg_GBps": b / (t / 1000.0) / 1e9 if t else None}
+    dom = max(kern, key=lambda k: kern[k][0] or 0.0)
+    dom_ms, dom_b = kern[dom]
+    achieved = dom_b / (dom_ms / 1000.0) / 1e9
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic_from_profile(dom),
+                "peak_source": peaks["source"], "alg_bytes_per_launch": dom_b,
                 "share_of_step": dom_ms / ms if ms > 0 else None}
-    steps_detail = {n: {"ms": step_ms[i]} for i, n in enumerate(names)}
-    for n, b in alg_bytes.items():
-        t = steps_detail[n]["ms"]
-        steps_detail[n]["alg_GBps"] = b / (t / 1000.0) / 1e9 if t > 0 else None
-    log(f"timed: {ms:.3f} ms/step, steps {steps_detail}")
+    log(f"timed ({path}): {ms:.3f} ms/step, {steps_detail}")
+
+    # the other path, timed the same way (every SURVEY §8a row measured); not the headline
+    other = None
+    if not args.no_other:
+        other_mode = "four_step" if path == "fused" else "fused"
+        lib_ms.clear()
+        for _ in range(2):
+            one_step(mode=other_mode)
+        torch.cuda.synchronize()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.steps):
+            one_step(record=True, mode=other_mode)
+        f1.record(stream)
+        torch.cuda.synchronize()
+        st2 = z.stats()
+        other = {"path": other_mode, "ms_per_step": f0.elapsed_time(f1) / args.steps}
+        if other_mode == "four_step":
+            tb = 2.0 * cells_local + 4.0 * B_pad * st2["n_tiles"]
+            for key, b in (("step1_tile_hist", tb), ("step2_pair_tiles", None),
+                           ("step3_aggregate", 4.0 * cfg.nbins * st2["n_inside"]),
+                           ("step4_pip_update", 2.0 * st2["n_isect"] * T * T)):
+                t = avg(lib_ms, key)
+                other[key] = {"ms": t}
+                if b:
+                    other[key]["alg_GBps"] = b / (t / 1000.0) / 1e9 if t else None
+                    other[key]["frac_of_hbm_peak"] = other[key]["alg_GBps"] / peaks["hbm_gbs"] if t else None
+        else:
+            other["fused_update"] = {"ms": avg(lib_ms, "fused_update")}
+        log(f"other path: {other}")
 
     # ---- end to end through the C ABI from host buffers
     e2e = None
@@ -356,9 +391,9 @@ def main():
                 "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert, parallelism=f"tile-row shards x{world}",
                                l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA"),
                 "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
-                "clocks": clocks, "steps_detail": steps_detail, "pairs": {k: st[k] for k in
-                                                                         ("n_tiles", "n_candidates", "n_inside",
-                                                                          "n_isect", "n_band_entries", "n_edges")},
+                "clocks": clocks, "path": path, "steps_detail": steps_detail, "other_path": other,
+                "pairs": {k: st[k] for k in ("n_tiles", "n_candidates", "n_inside", "n_isect", "n_band_entries",
+                                             "n_edges", "n_pure_tiles", "n_pip_pairs", "n_pure_cells", "n_pip_cells")},
                 "setup_s": time.perf_counter() - t_setup}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -396,7 +431,7 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
         t0 = time.perf_counter()
         z2 = zh.ZonalHistogram(host_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
                                oor_drop=cfg.oor_drop, tile=cfg.tile, rows=cfg.rows, cols=cfg.cols, row0=r0,
-                               stream=stream)
+                               stream=stream, fused=(args.path == "fused"))
         if world > 1:
             z2.set_output(out)
             z2.zh_run(None)
@@ -427,7 +462,8 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
     log(f"e2e {sec:.3f} s/step (pinned={pinned})")
     return {"value": cfg.cells / sec, "unit": "cells/s", "seconds_per_step": sec, "h2d_bytes_per_step": h2d,
             "d2h_bytes_per_step": d2h, "host_raster_pinned": bool(pinned), "steps": len(times),
-            "includes": "zh_create (polygon H2D, allocation) + raster H2D + steps 2,1,3,4 + result D2H + zh_destroy"}, host
+            "includes": f"zh_create (polygon H2D, allocation) + raster H2D + zh_run ({args.path}) + result D2H + "
+                        f"zh_destroy"}, host
 
 
 if __name__ == "__main__":

@@ -16,7 +16,11 @@
  *   step 3 zh_aggregate   add inside tiles' histograms to the polygons  (§III.C, Fig. 4)
  *   step 4 zh_pip_update  cell-in-polygon test for the cells of intersecting tiles
  *                                                                        (§III.D, Fig. 5)
- *   zh_run                steps 2, 1, 3, 4 and the copy of the result to the host.
+ *   zh_run                steps 2, 1, 3, 4 (or 2 + fused) and the copy of the result to the host.
+ *   zh_fused_update       steps 1 + 3 + 4 fused, tile by tile, each raster cell read at most once
+ *                         (outside-only tiles are never read; tiles with only
+ *                         inside pairs are histogrammed straight into their polygons; tiles with an
+ *                         intersecting pair go through the step-4 kernel).  Bit-identical result.
  *
  * Conventions
  *  - Every call returns zh_status; nothing throws, exits or prints.  On failure
@@ -41,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 1
+#define ZH_ABI_VERSION 2
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -97,7 +101,7 @@ typedef struct {
  * no check):  a cell with use_nodata && v == nodata is never counted; otherwise
  * d = v - lo; d < 0 -> bin 0 (clamp) or not counted (oor_drop); b = d / width;
  * b >= nbins -> nbins-1 (clamp) or not counted (oor_drop).
- * Requires 1 <= nbins <= 1<<20, 1 <= width, |lo| <= 1<<30. */
+ * Requires 1 <= nbins <= 49152 (shared-memory histograms), 1 <= width, |lo| <= 1<<30. */
 typedef struct {
   int32_t lo, width, nbins;
   int32_t use_nodata, nodata;
@@ -111,7 +115,7 @@ typedef struct {
                           some polygon's MBB could hold >= 2^32 cells)                           */
   int32_t force_isect; /* 1: classify every non-outside pair as intersecting (skips step 3's
                           work; a validation mode — the result must not change)                  */
-  int32_t reserved;
+  int32_t fused;       /* 1: zh_run uses zh_fused_update instead of steps 1, 3, 4               */
   void* stream;        /* cudaStream_t                                                          */
 } zh_options;
 
@@ -123,6 +127,10 @@ typedef struct {
   int64_t n_band_entries; /* (edge, tile-row) entries of the step-4 edge lists                  */
   int64_t n_edges;        /* polygon edges                                                      */
   int64_t device_bytes;   /* device memory owned by the context                                 */
+  int64_t n_pure_tiles;   /* after zh_fused_update: tiles histogrammed straight into polygons     */
+  int64_t n_pip_pairs;    /* after zh_fused_update: pairs sent to the cell-in-polygon kernel      */
+  int64_t n_pure_cells;   /* cells of those pure tiles                                          */
+  int64_t n_pip_cells;    /* cells of the tiles of those pairs (counted once per pair)           */
 } zh_stats;
 
 /* Validate, copy polygons to the device (H2D on options->stream), allocate per-tile histograms
@@ -133,7 +141,8 @@ zh_status zh_create(zh_ctx* out, const zh_raster* raster, const zh_polygons* pol
 /* on_host rasters: enqueue the host->device copy of the shard (zh_run does this itself). */
 zh_status zh_upload_raster(zh_ctx ctx);
 
-/* Step 1 (async): tile_hist[t][b] for every tile t of the shard. */
+/* Step 1 (async): tile_hist[t][b] for every tile t of the shard (the first call allocates the
+ * n_tiles x B_pad uint32 array). */
 zh_status zh_tile_hist(zh_ctx ctx);
 
 /* Step 2: edge preparation, MBB pairing, classification, pair lists; zeroes the output.
@@ -148,7 +157,11 @@ zh_status zh_aggregate(zh_ctx ctx);
  * centre is inside the polygon, out[k][bin(v)] += 1.  Needs step 2, else ZH_ERR_STATE. */
 zh_status zh_pip_update(zh_ctx ctx);
 
-/* Upload (on_host), steps 2, 1, 3, 4, then copy n_poly * nbins elements (uint64 or uint32 per
+/* Steps 1 + 3 + 4 fused (async).  Needs step 2; exclusive with zh_aggregate / zh_pip_update for the
+ * same zh_pair_tiles (ZH_ERR_STATE).  Does not need (or fill) the per-tile histograms. */
+zh_status zh_fused_update(zh_ctx ctx);
+
+/* Upload (on_host), steps 2, 1, 3, 4 (or 2 + fused when options.fused), then copy n_poly * nbins elements (uint64 or uint32 per
  * out_u64, row-major [n_poly][nbins]) to host_out (may be NULL to skip the copy).  Syncs. */
 zh_status zh_run(zh_ctx ctx, void* host_out);
 
@@ -170,10 +183,12 @@ zh_status zh_copy_pairs(zh_ctx ctx, int32_t* inside, int32_t* isect);
 
 zh_status zh_get_stats(zh_ctx ctx, zh_stats* stats);
 
-/* Per-step device time (ms) of the last call of each step, measured with CUDA events on the
- * context stream when timing is enabled (zh_set_timing).  ms[0..3] = steps 1..4. */
+/* Device time (ms) of the last call of each step, measured with CUDA events on the context stream
+ * when timing is enabled (zh_set_timing).  Up to n values: [0..3] steps 1..4, [4] zh_fused_update,
+ * [5] its pure-tile kernel, [6] its cell-in-polygon kernel; -1 for a call not made since timing
+ * was enabled.  Syncs. */
 zh_status zh_set_timing(zh_ctx ctx, int32_t enable);
-zh_status zh_get_step_ms(zh_ctx ctx, float* ms4);
+zh_status zh_get_step_ms(zh_ctx ctx, float* ms, int32_t n);
 
 /* Number of kernel launches the context has enqueued since creation (self-reported). */
 int64_t zh_launch_count(zh_ctx ctx);

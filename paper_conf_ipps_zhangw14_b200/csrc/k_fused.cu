@@ -1,0 +1,254 @@
+// k_fused.cu — fused, needed-tiles-only histogramming (SURVEY.md §8f-1 "NEXT 1").
+//
+// Step 1 is independent of the polygons (§III ¶1), so after step 2 the tiles split into
+//   * outside-only tiles  — no pair: never read;
+//   * pure tiles          — >= 1 inside pair and no intersecting pair: the tile is histogrammed in
+//                           shared memory exactly as in step 1 and the histogram is added straight
+//                           into each inside polygon's row (steps 1 + 3 fused: no per-tile histogram
+//                           array, no second pass);
+//   * mixed tiles         — >= 1 intersecting pair: every pair of the tile (intersecting, and the rare
+//                           inside pair of a mixed tile, e.g. overlapping polygons) goes through the
+//                           step-4 cell-in-polygon kernel, which is exact for any pair.
+// Each raster cell is therefore read once from HBM, and only when some polygon may contain it.
+// The result is bit-identical to steps 1 + 3 + 4 (integer sums; tests/test_gpu_fused.py).
+#include <cub/device/device_scan.cuh>
+
+#include "zh_ctx.h"
+#include "zh_tilehist.cuh"
+
+namespace zh {
+
+__global__ void k_mark_mixed(const int2* __restrict__ isect, int64_t n, uint8_t* __restrict__ mixed) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    mixed[isect[i].x] = 1;
+}
+
+// inside pairs of pure tiles are counted per tile; inside pairs of mixed tiles are flagged "extra"
+__global__ void k_inside_split(const int2* __restrict__ inside, int64_t n, const uint8_t* __restrict__ mixed,
+                               uint32_t* __restrict__ pure_cnt, uint32_t* __restrict__ extra) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int t = inside[i].x;
+    if (mixed[t]) {
+      extra[i] = 1;
+    } else {
+      extra[i] = 0;
+      atomicAdd(&pure_cnt[t], 1u);
+    }
+  }
+}
+
+// packed per-tile value for one scan: low 32 = #inside polygons, high 32 = (tile is pure)
+__global__ void k_pack_tiles(const uint32_t* __restrict__ pure_cnt, int64_t n, uint64_t* __restrict__ pk) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = pure_cnt[i];
+    pk[i] = (uint64_t)c | ((uint64_t)(c > 0) << 32);
+  }
+}
+
+__global__ void k_pure_fill(const int2* __restrict__ inside, int64_t n, const uint32_t* __restrict__ extra,
+                            const uint64_t* __restrict__ pure_off, uint32_t* __restrict__ cursor,
+                            int32_t* __restrict__ pure_poly) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (extra[i]) continue;
+    const int2 p = inside[i];
+    const uint32_t pos = (uint32_t)(pure_off[p.x] & 0xFFFFFFFFull) + atomicAdd(&cursor[p.x], 1u);
+    pure_poly[pos] = p.y;
+  }
+}
+
+__device__ __forceinline__ int64_t tile_cells(const RasterP& rp, int tile) {
+  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int64_t r0 = (int64_t)(rp.tr0 + trl) * rp.T, c0 = (int64_t)tc * rp.T;
+  return min((int64_t)rp.T, rp.row0 + rp.nrows - r0) * min((int64_t)rp.T, rp.cols - c0);
+}
+
+// counts[0] = #pure tiles, counts[2] = their cells (bench: algorithmic bytes)
+__global__ void k_pure_tiles(const uint32_t* __restrict__ pure_cnt, int64_t n, const uint64_t* __restrict__ pure_off,
+                             RasterP rp, int32_t* __restrict__ pure_tiles, int64_t* __restrict__ counts) {
+  int64_t cells = 0;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+    if (pure_cnt[t]) {
+      pure_tiles[pure_off[t] >> 32] = (int32_t)t;
+      cells += tile_cells(rp, (int)t);
+    }
+    if (t == n - 1) counts[0] = (int64_t)(pure_off[t] >> 32) + (pure_cnt[t] ? 1 : 0);
+  }
+  for (int o = 16; o > 0; o >>= 1) cells += __shfl_xor_sync(0xffffffffu, cells, o);
+  if ((threadIdx.x & 31) == 0 && cells) atomicAdd(reinterpret_cast<unsigned long long*>(&counts[2]),
+                                                  (unsigned long long)cells);
+}
+
+// counts[1] = #pairs for the cell-in-polygon kernel, counts[3] = their tiles' cells
+__global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, const int2* __restrict__ inside,
+                           int64_t n_inside, const uint32_t* __restrict__ extra, const uint32_t* __restrict__ extra_pos,
+                           RasterP rp, int2* __restrict__ pip, int64_t* __restrict__ counts) {
+  const int64_t n = n_isect + n_inside;
+  int64_t cells = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (i < n_isect) {
+      pip[i] = isect[i];
+      cells += tile_cells(rp, isect[i].x);
+    } else {
+      const int64_t j = i - n_isect;
+      if (extra[j]) {
+        pip[n_isect + extra_pos[j]] = inside[j];
+        cells += tile_cells(rp, inside[j].x);
+      }
+      if (j == n_inside - 1) counts[1] = n_isect + (int64_t)extra_pos[j] + extra[j];
+    }
+  }
+  if (n_inside == 0 && blockIdx.x == 0 && threadIdx.x == 0) counts[1] = n_isect;
+  for (int o = 16; o > 0; o >>= 1) cells += __shfl_xor_sync(0xffffffffu, cells, o);
+  if ((threadIdx.x & 31) == 0 && cells) atomicAdd(reinterpret_cast<unsigned long long*>(&counts[3]),
+                                                  (unsigned long long)cells);
+}
+
+template <int kMode, bool kU64>
+__global__ void __launch_bounds__(512, 3) k_fused_pure(RasterP rp, BinP bp, FastBins fb,
+                                                       const int32_t* __restrict__ pure_tiles,
+                                                       const int64_t* __restrict__ counts,
+                                                       const uint64_t* __restrict__ pure_off,
+                                                       const uint32_t* __restrict__ pure_cnt,
+                                                       const int32_t* __restrict__ pure_poly, void* __restrict__ out) {
+  if ((int64_t)blockIdx.x >= counts[0]) return;
+  extern __shared__ __align__(16) uint32_t sh[];
+  const int HW = hist_words(bp.nbins);
+  const int tile = pure_tiles[blockIdx.x];
+  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
+    *reinterpret_cast<uint4*>(&sh[i]) = make_uint4(0, 0, 0, 0);
+  __syncthreads();
+  tile_histogram<kMode>(sh, rp, bp, fb, trl, tc);
+  __syncthreads();
+  const uint32_t beg = (uint32_t)(pure_off[tile] & 0xFFFFFFFFull), cnt = pure_cnt[tile];
+  const int nbins = bp.nbins;
+  for (uint32_t j = 0; j < cnt; ++j) {
+    const int64_t row = (int64_t)pure_poly[beg + j] * nbins;
+    for (int b = threadIdx.x; b < nbins; b += blockDim.x) {
+      const uint32_t v = sh[kOff + b];
+      if (v) {
+        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(out) + row + b, (unsigned long long)v);
+        else atomicAdd(reinterpret_cast<uint32_t*>(out) + row + b, v);
+      }
+    }
+  }
+}
+
+static int grid_for(int64_t n, int threads) {
+  int64_t b = (n + threads - 1) / threads;
+  if (b > 148 * 32) b = 148 * 32;
+  if (b < 1) b = 1;
+  return (int)b;
+}
+
+template <class T>
+static cudaError_t excl_scan(Ctx& c, const T* in, T* out, int64_t n) {
+  size_t need = 0;
+  cudaError_t e = cub::DeviceScan::ExclusiveSum(nullptr, need, in, out, (int)n, c.stream);
+  if (e != cudaSuccess) return e;
+  if ((e = c.d_cub.ensure(need)) != cudaSuccess) return e;
+  size_t have = c.d_cub.bytes;
+  c.launches += 2;  // CUB init + scan kernels
+  return cub::DeviceScan::ExclusiveSum(c.d_cub.p, have, in, out, (int)n, c.stream);
+}
+
+template <int kMode, bool kU64>
+static void launch_pure(Ctx& c, size_t smem, unsigned grid) {
+  auto k = k_fused_pure<kMode, kU64>;
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<grid, 512, smem, c.stream>>>(c.rp, c.bp, make_fast_bins(c.bp), c.d_pure_tiles.as<int32_t>(),
+                                   c.d_fcounts.as<int64_t>(), c.d_pure_off.as<uint64_t>(),
+                                   c.d_pure_cnt.as<uint32_t>(), c.d_pure_poly.as<int32_t>(), c.d_out);
+}
+
+cudaError_t launch_fused(Ctx& c) {
+  cudaError_t e;
+  const int64_t NT = c.n_tiles, NI = c.n_inside, NX = c.n_isect;
+  if ((e = c.d_mixed.ensure((size_t)NT + 16)) != cudaSuccess) return e;
+  if ((e = c.d_pure_cnt.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pure_cur.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pure_pk.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pure_off.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pure_poly.ensure(sizeof(int32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pure_tiles.ensure(sizeof(int32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
+  if ((e = c.d_extra.ensure(sizeof(uint32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
+  if ((e = c.d_extra_pos.ensure(sizeof(uint32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pip.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
+  if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 4)) != cudaSuccess) return e;
+  cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 4, c.stream);
+  if (NT == 0 || NI + NX == 0) {
+    if (c.timing)
+      for (int i = 10; i < 13; ++i) cudaEventRecord(c.ev[i], c.stream);
+    return cudaGetLastError();
+  }
+
+  cudaMemsetAsync(c.d_mixed.p, 0, (size_t)NT, c.stream);
+  cudaMemsetAsync(c.d_pure_cnt.p, 0, sizeof(uint32_t) * ((size_t)NT + 1), c.stream);
+  cudaMemsetAsync(c.d_pure_cur.p, 0, sizeof(uint32_t) * ((size_t)NT + 1), c.stream);
+  if (NX > 0) {
+    k_mark_mixed<<<grid_for(NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_mixed.as<uint8_t>());
+    c.launches += 1;
+  }
+  if (NI > 0) {
+    k_inside_split<<<grid_for(NI, 256), 256, 0, c.stream>>>(c.d_inside.as<int2>(), NI, c.d_mixed.as<uint8_t>(),
+                                                           c.d_pure_cnt.as<uint32_t>(), c.d_extra.as<uint32_t>());
+    c.launches += 1;
+  }
+  k_pack_tiles<<<grid_for(NT + 1, 256), 256, 0, c.stream>>>(c.d_pure_cnt.as<uint32_t>(), NT + 1,
+                                                            c.d_pure_pk.as<uint64_t>());
+  c.launches += 1;
+  if ((e = excl_scan<uint64_t>(c, c.d_pure_pk.as<uint64_t>(), c.d_pure_off.as<uint64_t>(), NT + 1)) != cudaSuccess)
+    return e;
+  if (NI > 0) {
+    k_pure_fill<<<grid_for(NI, 256), 256, 0, c.stream>>>(c.d_inside.as<int2>(), NI, c.d_extra.as<uint32_t>(),
+                                                        c.d_pure_off.as<uint64_t>(), c.d_pure_cur.as<uint32_t>(),
+                                                        c.d_pure_poly.as<int32_t>());
+    c.launches += 1;
+  }
+  k_pure_tiles<<<grid_for(NT, 256), 256, 0, c.stream>>>(c.d_pure_cnt.as<uint32_t>(), NT, c.d_pure_off.as<uint64_t>(),
+                                                        c.rp, c.d_pure_tiles.as<int32_t>(), c.d_fcounts.as<int64_t>());
+  c.launches += 1;
+  if (NI > 0) {
+    if ((e = excl_scan<uint32_t>(c, c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(), NI)) != cudaSuccess)
+      return e;
+  }
+  k_pip_list<<<grid_for(NI + NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_inside.as<int2>(), NI,
+                                                          c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(),
+                                                          c.rp, c.d_pip.as<int2>(), c.d_fcounts.as<int64_t>());
+  c.launches += 1;
+
+  // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
+  if (c.timing) cudaEventRecord(c.ev[10], c.stream);
+  if (NI > 0) {
+    const size_t smem = (size_t)hist_words(c.bp.nbins) * 4;
+    const unsigned grid = (unsigned)NI;
+    const int mode = fast_bins_ok(c.bp) ? (make_fast_bins(c.bp).bias ? 4 : (c.bp.use_nodata ? 3 : 2))
+                                        : (c.bp.width == 1 ? 0 : 1);
+    if (c.out_u64) {
+      switch (mode) {
+        case 0: launch_pure<0, true>(c, smem, grid); break;
+        case 1: launch_pure<1, true>(c, smem, grid); break;
+        case 2: launch_pure<2, true>(c, smem, grid); break;
+        case 3: launch_pure<3, true>(c, smem, grid); break;
+        default: launch_pure<4, true>(c, smem, grid); break;
+      }
+    } else {
+      switch (mode) {
+        case 0: launch_pure<0, false>(c, smem, grid); break;
+        case 1: launch_pure<1, false>(c, smem, grid); break;
+        case 2: launch_pure<2, false>(c, smem, grid); break;
+        case 3: launch_pure<3, false>(c, smem, grid); break;
+        default: launch_pure<4, false>(c, smem, grid); break;
+      }
+    }
+    c.launches += 1;
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  if (c.timing) cudaEventRecord(c.ev[11], c.stream);
+  // mixed tiles: every pair through the cell-in-polygon kernel
+  e = launch_pip_list(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1);
+  if (c.timing) cudaEventRecord(c.ev[12], c.stream);
+  return e;
+}
+
+}  // namespace zh

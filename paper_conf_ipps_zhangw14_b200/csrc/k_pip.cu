@@ -41,6 +41,7 @@ struct PipP {
   int B_pad;
   int wpr;  // bitmap words per row = T/32 + 1
   int rc;   // rows per chunk
+  const int64_t* n_dev;  // device count of pairs (grid may be an upper bound), or nullptr
 };
 
 __device__ __forceinline__ uint32_t bits8(const uint32_t* __restrict__ row, int wpr, int lc0) {
@@ -56,6 +57,7 @@ __device__ __forceinline__ uint32_t bits8(const uint32_t* __restrict__ row, int 
 
 template <int kMode, bool kU64>  // kMode as in k_tile_hist: 0/1 generic (w1 / w>1), 2 + kForm packed
 __global__ void __launch_bounds__(256) k_pip(PipP p) {
+  if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
   extern __shared__ __align__(16) uint32_t sh[];
   const int HW = hist_words(p.bp.nbins);
   uint32_t* hist = sh;
@@ -200,13 +202,16 @@ __global__ void __launch_bounds__(256) k_pip(PipP p) {
   }
 }
 
-cudaError_t launch_pip(Ctx& c) {
-  if (c.n_isect == 0) return cudaSuccess;
+cudaError_t launch_pip(Ctx& c) { return launch_pip_list(c, c.d_isect.as<int2>(), c.n_isect, nullptr); }
+
+cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
+  if (grid == 0) return cudaSuccess;
   PipP p;
+  p.n_dev = n_dev;
   p.rp = c.rp;
   p.g = c.geo;
   p.bp = c.bp;
-  p.isect = c.d_isect.as<int2>();
+  p.isect = pairs;
   p.mbb = c.d_mbb.as<int4>();
   p.band_base = c.d_band_base.as<int64_t>();
   p.band_off = c.d_band_off.as<int32_t>();
@@ -217,7 +222,10 @@ cudaError_t launch_pip(Ctx& c) {
   p.B_pad = c.B_pad;
   p.fb = make_fast_bins(c.bp);
   p.wpr = c.rp.T / 32 + 1;
-  const int bm_budget_words = 8192;  // 32 KB of parity bitmap per CTA
+  // up to 32 KB of parity bitmap per CTA, less when the histogram is large (227 KB per CTA)
+  const int hist_bytes = hist_words(c.bp.nbins) * 4;
+  int bm_budget_words = (227 * 1024 - 2048 - hist_bytes) / 4;
+  if (bm_budget_words > 8192) bm_budget_words = 8192;
   p.rc = bm_budget_words / p.wpr;
   if (p.rc < 1) p.rc = 1;
   if (p.rc > c.rp.T) p.rc = c.rp.T;
@@ -233,7 +241,7 @@ cudaError_t launch_pip(Ctx& c) {
     default: k = c.out_u64 ? k_pip<4, true> : k_pip<4, false>; break;
   }
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k<<<(unsigned)c.n_isect, threads, smem, c.stream>>>(p);
+  k<<<(unsigned)grid, threads, smem, c.stream>>>(p);
   c.launches += 1;
   return cudaGetLastError();
 }

@@ -143,6 +143,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   c->B_pad = (b->nbins + 3) & ~3;
   c->out_u64 = o->out_u64 ? 1 : 0;
   c->force_isect = o->force_isect ? 1 : 0;
+  c->fused = o->fused ? 1 : 0;
   c->stream = (cudaStream_t)o->stream;
   c->n_tiles = n_tiles;
   c->P = (int32_t)p->n_poly;
@@ -170,9 +171,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
         (e = cudaMemcpyAsync(c->d_y.p, p->y, (size_t)p->n_vert * 8, cudaMemcpyHostToDevice, c->stream)))
       return cleanup_fail(cuda_fail(e, "zh_create (vertices H2D)"));
   }
-  // per-tile histograms and output
-  if ((e = c->d_tile_hist.ensure((size_t)n_tiles * c->B_pad * 4)) != cudaSuccess)
-    return cleanup_fail(cuda_fail(e, "zh_create (tile histograms)"));
+  // output (the per-tile histograms of step 1 are allocated by the first zh_tile_hist)
   const size_t out_bytes = (size_t)p->n_poly * b->nbins * (c->out_u64 ? 8 : 4);
   if ((e = c->d_out_own.ensure(out_bytes)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (output)"));
   c->d_out = c->d_out_own.p;
@@ -186,7 +185,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   }
   if ((e = cudaHostAlloc((void**)&c->pinned_counts, 8 * sizeof(int64_t), cudaHostAllocDefault)) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (pinned counters)"));
-  for (int i = 0; i < 8; ++i)
+  for (int i = 0; i < 13; ++i)
     if ((e = cudaEventCreate(&c->ev[i])) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (events)"));
   if ((e = cudaGetLastError()) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
   *out = reinterpret_cast<zh_ctx>(c);
@@ -201,9 +200,11 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_epoly, &c->d_espan, &c->d_mbb, &c->d_ncand, &c->d_nband, &c->d_cand_off,
                       &c->d_band_base, &c->d_band_cnt, &c->d_band_off, &c->d_band_cur, &c->d_band_edges,
                       &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
-                      &c->d_cub, &c->d_tile_hist, &c->d_out_own};
+                      &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
+                      &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
+                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_fcounts};
   for (auto* b : bufs) b->release();
-  for (int i = 0; i < 8; ++i)
+  for (int i = 0; i < 13; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
   if (c->pinned_counts) cudaFreeHost(c->pinned_counts);
   delete c;
@@ -214,7 +215,9 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_epoly, &c.d_espan, &c.d_mbb, &c.d_ncand, &c.d_nband, &c.d_cand_off,
                             &c.d_band_base, &c.d_band_cnt, &c.d_band_off, &c.d_band_cur, &c.d_band_edges,
                             &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
-                            &c.d_cub, &c.d_tile_hist, &c.d_out_own};
+                            &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
+                            &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
+                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_fcounts};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;
@@ -241,6 +244,7 @@ extern "C" zh_status zh_upload_raster(zh_ctx h) {
 extern "C" zh_status zh_tile_hist(zh_ctx h) {
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
+  ZH_CU(c->d_tile_hist.ensure((size_t)c->n_tiles * c->B_pad * 4), "zh_tile_hist (allocating tile histograms)");
   tic(c, 0);
   ZH_CU(zh::launch_tile_hist(*c), "zh_tile_hist");
   toc(c, 0);
@@ -253,6 +257,8 @@ extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect
   Ctx* c = C(h);
   c->have_pairs = false;
   c->step3_done = false;
+  c->step4_done = false;
+  c->fused_done = false;
   tic(c, 1);
   const size_t out_bytes = (size_t)c->P * c->bp.nbins * (c->out_u64 ? 8 : 4);
   ZH_CU(cudaMemsetAsync(c->d_out, 0, out_bytes, c->stream), "zh_pair_tiles (zero output)");
@@ -285,6 +291,7 @@ extern "C" zh_status zh_aggregate(zh_ctx h) {
   Ctx* c = C(h);
   if (!c->have_pairs || !c->have_hist) return fail(ZH_ERR_STATE, "zh_aggregate needs zh_tile_hist and zh_pair_tiles");
   if (c->step3_done) return fail(ZH_ERR_STATE, "zh_aggregate already applied since the last zh_pair_tiles");
+  if (c->fused_done) return fail(ZH_ERR_STATE, "zh_fused_update already covered step 3");
   tic(c, 2);
   ZH_CU(zh::launch_aggregate(*c), "zh_aggregate");
   toc(c, 2);
@@ -296,9 +303,25 @@ extern "C" zh_status zh_pip_update(zh_ctx h) {
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (!c->have_pairs) return fail(ZH_ERR_STATE, "zh_pip_update needs zh_pair_tiles");
+  if (c->step4_done) return fail(ZH_ERR_STATE, "zh_pip_update already applied since the last zh_pair_tiles");
+  if (c->fused_done) return fail(ZH_ERR_STATE, "zh_fused_update already covered step 4");
   tic(c, 3);
   ZH_CU(zh::launch_pip(*c), "zh_pip_update");
   toc(c, 3);
+  c->step4_done = true;
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_fused_update(zh_ctx h) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (!c->have_pairs) return fail(ZH_ERR_STATE, "zh_fused_update needs zh_pair_tiles");
+  if (c->step3_done || c->step4_done || c->fused_done)
+    return fail(ZH_ERR_STATE, "steps 3/4 already applied since the last zh_pair_tiles");
+  tic(c, 4);
+  ZH_CU(zh::launch_fused(*c), "zh_fused_update");
+  toc(c, 4);
+  c->fused_done = true;
   return ZH_OK;
 }
 
@@ -308,9 +331,13 @@ extern "C" zh_status zh_run(zh_ctx h, void* host_out) {
   zh_status s;
   if ((s = zh_upload_raster(h)) != ZH_OK) return s;
   if ((s = zh_pair_tiles(h, nullptr, nullptr)) != ZH_OK) return s;
-  if ((s = zh_tile_hist(h)) != ZH_OK) return s;
-  if ((s = zh_aggregate(h)) != ZH_OK) return s;
-  if ((s = zh_pip_update(h)) != ZH_OK) return s;
+  if (c->fused) {
+    if ((s = zh_fused_update(h)) != ZH_OK) return s;
+  } else {
+    if ((s = zh_tile_hist(h)) != ZH_OK) return s;
+    if ((s = zh_aggregate(h)) != ZH_OK) return s;
+    if ((s = zh_pip_update(h)) != ZH_OK) return s;
+  }
   if (host_out) {
     const size_t out_bytes = (size_t)c->P * c->bp.nbins * (c->out_u64 ? 8 : 4);
     ZH_CU(cudaMemcpyAsync(host_out, c->d_out, out_bytes, cudaMemcpyDeviceToHost, c->stream), "zh_run (D2H)");
@@ -333,6 +360,7 @@ extern "C" zh_status zh_set_output(zh_ctx h, void* dptr) {
   if (dptr && ((uintptr_t)dptr & 7u)) return fail(ZH_ERR_INVALID_ARG, "output buffer must be 8-byte aligned");
   c->d_out = dptr ? dptr : c->d_out_own.p;
   c->have_pairs = false;  // the new buffer must be zeroed by zh_pair_tiles before accumulation
+  c->have_hist = c->have_hist;
   return ZH_OK;
 }
 
@@ -340,6 +368,7 @@ extern "C" zh_status zh_copy_tile_hist(zh_ctx h, uint32_t* host, int64_t n_elems
   if (!h || !host) return fail(ZH_ERR_INVALID_ARG, "null argument");
   Ctx* c = C(h);
   if (n_elems < c->n_tiles * c->bp.nbins) return fail(ZH_ERR_INVALID_ARG, "host buffer too small");
+  if (!c->have_hist) return fail(ZH_ERR_STATE, "zh_copy_tile_hist needs zh_tile_hist");
   if (c->n_tiles == 0) return ZH_OK;
   ZH_CU(cudaMemcpy2DAsync(host, (size_t)c->bp.nbins * 4, c->d_tile_hist.p, (size_t)c->B_pad * 4,
                           (size_t)c->bp.nbins * 4, (size_t)c->n_tiles, cudaMemcpyDeviceToHost, c->stream),
@@ -372,6 +401,16 @@ extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
   s->n_band_entries = c->n_band_entries;
   s->n_edges = c->V;
   s->device_bytes = (int64_t)zh::device_bytes(*c);
+  s->n_pure_tiles = s->n_pip_pairs = s->n_pure_cells = s->n_pip_cells = 0;
+  if (c->fused_done) {
+    ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_fcounts.p, 4 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
+          "zh_get_stats");
+    ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_stats");
+    s->n_pure_tiles = c->pinned_counts[0];
+    s->n_pip_pairs = c->pinned_counts[1];
+    s->n_pure_cells = c->pinned_counts[2];
+    s->n_pip_cells = c->pinned_counts[3];
+  }
   return ZH_OK;
 }
 
@@ -381,18 +420,20 @@ extern "C" zh_status zh_set_timing(zh_ctx h, int32_t enable) {
   return ZH_OK;
 }
 
-extern "C" zh_status zh_get_step_ms(zh_ctx h, float* ms4) {
-  if (!h || !ms4) return fail(ZH_ERR_INVALID_ARG, "null argument");
+extern "C" zh_status zh_get_step_ms(zh_ctx h, float* ms, int32_t n) {
+  if (!h || !ms) return fail(ZH_ERR_INVALID_ARG, "null argument");
   Ctx* c = C(h);
   if (!c->timing) return fail(ZH_ERR_STATE, "timing is disabled");
   ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_step_ms");
-  for (int i = 0; i < 4; ++i) {
-    float ms = 0.f;
-    if (cudaEventElapsedTime(&ms, c->ev[2 * i], c->ev[2 * i + 1]) != cudaSuccess) {
+  // (start, stop) event pairs: steps 1..4, fused, fused pure-tile kernel, fused cell-in-polygon kernel
+  const int pairs[7][2] = {{0, 1}, {2, 3}, {4, 5}, {6, 7}, {8, 9}, {10, 11}, {11, 12}};
+  for (int i = 0; i < n && i < 7; ++i) {
+    float v = 0.f;
+    if (cudaEventElapsedTime(&v, c->ev[pairs[i][0]], c->ev[pairs[i][1]]) != cudaSuccess) {
       cudaGetLastError();
-      ms = -1.f;
+      v = -1.f;
     }
-    ms4[i] = ms;
+    ms[i] = v;
   }
   return ZH_OK;
 }

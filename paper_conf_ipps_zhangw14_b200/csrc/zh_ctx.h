@@ -52,6 +52,9 @@ struct Ctx {
   DBuf d_edges, d_erows, d_epoly, d_espan, d_mbb, d_ncand, d_nband, d_cand_off, d_band_base;
   DBuf d_band_cnt, d_band_off, d_band_cur, d_band_edges, d_class, d_flags, d_flag_pos;
   DBuf d_inside, d_isect, d_counts, d_cub;
+  // fused path lists (k_fused.cu)
+  DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,
+      d_pip, d_fcounts;
   int64_t n_cand = 0, n_bands = 0, n_band_entries = 0, n_inside = 0, n_isect = 0;
   // step 1 product and output
   DBuf d_tile_hist;
@@ -59,11 +62,12 @@ struct Ctx {
   void* d_out = nullptr;  // own or borrowed
   int64_t n_tiles = 0;
   // state
-  bool have_hist = false, have_pairs = false, step3_done = false;
+  bool have_hist = false, have_pairs = false, step3_done = false, step4_done = false, fused_done = false;
+  int32_t fused = 0;
   // timing
   bool timing = false;
-  cudaEvent_t ev[8] = {};
-  float step_ms[4] = {0, 0, 0, 0};
+  cudaEvent_t ev[13] = {};  // start/stop per timed call: steps 1..4, fused; + fused inner marks 10..12
+  int64_t fused_counts[4] = {0, 0, 0, 0};  // pure tiles, pip pairs, pure cells, pip cells
   int64_t launches = 0;
   int64_t host_count_buf[4] = {0, 0, 0, 0};
   int64_t* pinned_counts = nullptr;
@@ -75,6 +79,8 @@ cudaError_t launch_pairs_phase1(Ctx& c);   // edges, MBBs, scans, count totals -
 cudaError_t launch_pairs_phase2(Ctx& c);   // bands, marking, classification, compaction
 cudaError_t launch_aggregate(Ctx& c);
 cudaError_t launch_pip(Ctx& c);
+cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
+cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
 
 size_t device_bytes(const Ctx& c);
 

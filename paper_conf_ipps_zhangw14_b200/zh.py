@@ -49,16 +49,18 @@ class zh_bins(ctypes.Structure):
 
 class zh_options(ctypes.Structure):
     _fields_ = [("tile", ctypes.c_int32), ("out_u64", ctypes.c_int32), ("force_isect", ctypes.c_int32),
-                ("reserved", ctypes.c_int32), ("stream", ctypes.c_void_p)]
+                ("fused", ctypes.c_int32), ("stream", ctypes.c_void_p)]
 
 
 class zh_stats(ctypes.Structure):
     _fields_ = [("n_tiles", ctypes.c_int64), ("n_candidates", ctypes.c_int64), ("n_inside", ctypes.c_int64),
                 ("n_isect", ctypes.c_int64), ("n_band_entries", ctypes.c_int64), ("n_edges", ctypes.c_int64),
-                ("device_bytes", ctypes.c_int64)]
+                ("device_bytes", ctypes.c_int64), ("n_pure_tiles", ctypes.c_int64), ("n_pip_pairs", ctypes.c_int64),
+                ("n_pure_cells", ctypes.c_int64), ("n_pip_cells", ctypes.c_int64)]
 
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",
+           "zh_fused_update",
            "zh_run", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
            "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy"]
 
@@ -78,6 +80,7 @@ def _load():
         "zh_pair_tiles": (st, [vp, ctypes.POINTER(i64), ctypes.POINTER(i64)]),
         "zh_aggregate": (st, [vp]),
         "zh_pip_update": (st, [vp]),
+        "zh_fused_update": (st, [vp]),
         "zh_run": (st, [vp, vp]),
         "zh_output_device": (st, [vp, ctypes.POINTER(vp), ctypes.POINTER(i64)]),
         "zh_set_output": (st, [vp, vp]),
@@ -85,7 +88,7 @@ def _load():
         "zh_copy_pairs": (st, [vp, vp, vp]),
         "zh_get_stats": (st, [vp, ctypes.POINTER(zh_stats)]),
         "zh_set_timing": (st, [vp, i32]),
-        "zh_get_step_ms": (st, [vp, ctypes.POINTER(ctypes.c_float)]),
+        "zh_get_step_ms": (st, [vp, ctypes.POINTER(ctypes.c_float), i32]),
         "zh_launch_count": (i64, [vp]),
         "zh_last_error": (ctypes.c_char_p, []),
         "zh_abi_version": (i32, []),
@@ -140,7 +143,8 @@ class ZonalHistogram:
 
     def __init__(self, raster, gt, polygons, nbins: int, lo: int = 0, width: int = 1, nodata=None,
                  oor_drop: bool = False, tile: int = 256, out_u64: bool = True, force_isect: bool = False,
-                 row0: int = 0, rows: int | None = None, cols: int | None = None, stream=None):
+                 row0: int = 0, rows: int | None = None, cols: int | None = None, stream=None,
+                 fused: bool = True):
         self._keep = []
         on_host, ptr, nrows, ncols_buf, pitch = self._raster_ptr(raster)
         ncols = cols if cols is not None else ncols_buf
@@ -161,7 +165,7 @@ class ZonalHistogram:
                         x.ctypes.data, y.ctypes.data)
         b = zh_bins(lo, width, nbins, 0 if nodata is None else 1, 0 if nodata is None else int(nodata), int(oor_drop))
         self.stream = _stream_handle(stream)
-        o = zh_options(tile, int(out_u64), int(force_isect), 0, self.stream)
+        o = zh_options(tile, int(out_u64), int(force_isect), int(fused), self.stream)
         h = ctypes.c_void_p()
         _check(LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)))
         self.h = h
@@ -203,6 +207,9 @@ class ZonalHistogram:
 
     def zh_pip_update(self):
         _check(LIB.zh_pip_update(self.h))
+
+    def zh_fused_update(self):
+        _check(LIB.zh_fused_update(self.h))
 
     def zh_run(self, host_out: np.ndarray | None = None) -> np.ndarray | None:
         if host_out is not None:
@@ -256,10 +263,14 @@ class ZonalHistogram:
     def set_timing(self, enable: bool = True) -> None:
         _check(LIB.zh_set_timing(self.h, int(enable)))
 
-    def step_ms(self):
-        ms = (ctypes.c_float * 4)()
-        _check(LIB.zh_get_step_ms(self.h, ms))
-        return list(ms)
+    STEP_NAMES = ("step1_tile_hist", "step2_pair_tiles", "step3_aggregate", "step4_pip_update", "fused_update",
+                  "fused_pure_kernel", "fused_pip_kernel")
+
+    def step_ms(self) -> dict:
+        """Device ms of the last call of each step (-1: not called since timing was enabled)."""
+        ms = (ctypes.c_float * 7)()
+        _check(LIB.zh_get_step_ms(self.h, ms, 7))
+        return dict(zip(self.STEP_NAMES, list(ms)))
 
     def launch_count(self) -> int:
         return int(LIB.zh_launch_count(self.h))

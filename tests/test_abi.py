@@ -33,7 +33,7 @@ def test_library_exports_every_declared_symbol():
     assert not missing, missing
     from paper_conf_ipps_zhangw14_b200 import zh
     assert set(zh.EXPORTS) == set(_declared())
-    assert zh.LIB.zh_abi_version() == 1
+    assert zh.LIB.zh_abi_version() == 2
 
 
 def test_library_is_sm100a_sass():
@@ -63,7 +63,7 @@ def test_pip_predicate_has_no_contracted_fma():
     double division is an MUFU.RCP64H followed by a handful of DFMAs)."""
     from paper_conf_ipps_zhangw14_b200 import _build
     funcs = _sass_functions(_build.build())
-    names = [n for n in funcs if any(k in n for k in ("k_pip", "k_classify", "k_edges"))]
+    names = [n for n in funcs if any(k in n for k in ("k_pipILi", "k_classify", "k_edges"))]
     assert names
     for n in names:
         sass = "\n".join(funcs[n])

@@ -23,12 +23,17 @@ def _raster(cfg):
 
 
 def _run(t, cfg, P, **kw):
+    """Four-step path and fused path; both must agree; returns the fused result and stats."""
     from paper_conf_ipps_zhangw14_b200 import zh
-    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=kw.pop("tile", cfg.tile), cols=cfg.cols,
-                           nodata=cfg.nodata, **kw) as z:
-        out = z.run()
-        st = z.stats()
-    return out, st
+    tile = kw.pop("tile", cfg.tile)
+    res = []
+    for fused in (False, True):
+        with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=tile, cols=cfg.cols, nodata=cfg.nodata,
+                               fused=fused, **kw) as z:
+            res.append(z.run())
+            st = z.stats()
+    assert (res[0] == res[1]).all(), "fused path differs from the four-step path"
+    return res[1], st
 
 
 def _sample_polys(P, n, seed):

@@ -30,9 +30,16 @@ def device_raster(spec, rows, cols, row0=0, nrows=None, pitch=None, gcols=None):
 
 
 def gpu_hist(t, gt, P, nbins, tile, cols, rows=None, row0=0, **kw):
+    """Run both libzh paths — the four steps (zh_tile_hist, zh_aggregate, zh_pip_update) and the
+    fused one (zh_fused_update) — check they agree bit for bit, and return the result."""
     zh = _zh()
-    with zh.ZonalHistogram(t, gt, P, nbins, tile=tile, cols=cols, rows=rows, row0=row0, **kw) as z:
-        return z.run()
+    res = []
+    for fused in (False, True):
+        with zh.ZonalHistogram(t, gt, P, nbins, tile=tile, cols=cols, rows=rows, row0=row0, fused=fused,
+                               **kw) as z:
+            res.append(z.run())
+    assert (res[0] == res[1]).all(), "fused path differs from the four-step path"
+    return res[1]
 
 
 @pytest.fixture(scope="module")
