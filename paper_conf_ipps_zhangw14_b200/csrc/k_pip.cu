@@ -22,6 +22,7 @@
 //     into a CTA-private shared histogram, flushed once per pair with one global atomic per
 //     non-zero bin (no race).
 #include "zh_ctx.h"
+#include "zh_parity.cuh"
 
 namespace zh {
 
@@ -44,43 +45,26 @@ struct PipP {
   const int64_t* n_dev;  // device count of pairs (grid may be an upper bound), or nullptr
 };
 
-__device__ __forceinline__ uint32_t bits8(const uint32_t* __restrict__ row, int wpr, int lc0) {
-  // parity bits of local columns lc0 .. lc0+7 (lc0 may be negative; missing bits -> 0)
-  if (lc0 >= 0) {
-    const int wi = lc0 >> 5, sh = lc0 & 31;
-    uint64_t v = row[wi];
-    if (sh > 24 && wi + 1 < wpr) v |= (uint64_t)row[wi + 1] << 32;
-    return (uint32_t)(v >> sh) & 0xFFu;
-  }
-  return (row[0] << (-lc0)) & 0xFFu;
-}
-
 template <int kMode, bool kU64>  // kMode as in k_tile_hist: 0/1 generic (w1 / w>1), 2 + kForm packed
 __global__ void __launch_bounds__(256) k_pip(PipP p) {
   if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
   extern __shared__ __align__(16) uint32_t sh[];
+  __shared__ LongQ lq;
   const int HW = hist_words(p.bp.nbins);
   uint32_t* hist = sh;
   uint32_t* bm = sh + HW;
+  if (threadIdx.x == 0) lq.n = 0;
   const RasterP& rp = p.rp;
   const Geo& g = p.g;
 
   const int2 pr = p.isect[blockIdx.x];
   const int tile = pr.x, k = pr.y;
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
-  const int tr = rp.tr0 + trl;
-  const int64_t r0 = (int64_t)tr * rp.T;
-  const int h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - r0);
-  const int64_t c0 = (int64_t)tc * rp.T;
-  const int w = (int)min((int64_t)rp.T, rp.cols - c0);
+  const TileGeom t = tile_geom(rp, g, tile);
+  const int64_t r0 = t.r0, c0 = t.c0;
+  const int h = t.h, w = t.w;
   const int4 m = p.mbb[k];
-  const int64_t band = p.band_base[k] + (tr - m.z);
+  const int64_t band = p.band_base[k] + ((int)(r0 / rp.T) - m.z);
   const int e0 = p.band_off[band], e1 = p.band_off[band + 1];
-  const bool s = g.gt1 > 0;
-  // centre-x range of the tile's columns, and half a cell of margin
-  const double xa_t = col_centre(g, c0), xb_t = col_centre(g, c0 + w - 1);
-  const double xlo_t = fmin(xa_t, xb_t), xhi_t = fmax(xa_t, xb_t);
-  const double half = 0.5 * fabs(g.gt1);
 
   for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
     *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
@@ -97,48 +81,8 @@ __global__ void __launch_bounds__(256) k_pip(PipP p) {
     const int64_t rlo = r0 + cr, rhi = rlo + ch;  // global rows of this chunk
     for (int i = threadIdx.x; i < ch * p.wpr; i += blockDim.x) bm[i] = 0;
     __syncthreads();
-    // ---- crossings: flips of the difference bitmap
-    for (int i = e0 + threadIdx.x; i < e1; i += blockDim.x) {
-      const int v = p.band_edges[i];
-      const int2 rr = p.erows[v];
-      const int64_t ra = max((int64_t)rr.x, rlo), rb = min((int64_t)rr.y, rhi);
-      if (ra >= rb) continue;
-      const Edge e = p.edges[v];
-      const double exl = fmin(e.xa, e.xb), exh = fmax(e.xa, e.xb);
-      if (exh + half < xlo_t) continue;  // xi < every xc: crosses no cell of the tile
-      if (exl - half > xhi_t) {          // xi > every xc: crosses every cell
-        for (int64_t r = ra; r < rb; ++r) {
-          const int lr = (int)(r - rlo);
-          atomicXor(&bm[lr * p.wpr + (w >> 5)], 1u << (w & 31));
-        }
-        continue;
-      }
-      for (int64_t r = ra; r < rb; ++r) {
-        const double yc = row_centre(g, r);
-        const double xi = intercept(e, yc);
-        const double est = (xi - g.gt0) / g.gt1 - 0.5 - (double)c0;
-        int64_t ei;
-        if (!(est > 0.0)) ei = 0;
-        else if (est > (double)w) ei = w;
-        else ei = (int64_t)ceil(est);
-        const int64_t jb = first_false(0, w, ei, [&](int64_t j) { return (col_centre(g, c0 + j) < xi) == s; });
-        const int lr = (int)(r - rlo);
-        if (jb > 0) atomicXor(&bm[lr * p.wpr + (int)(jb >> 5)], 1u << (jb & 31));
-        if (!s) atomicXor(&bm[lr * p.wpr + (w >> 5)], 1u << (w & 31));
-      }
-    }
-    __syncthreads();
-    // ---- suffix XOR: parity(lc) = XOR_{j > lc} D[j]
-    for (int lr = threadIdx.x; lr < ch; lr += blockDim.x) {
-      uint32_t* row = bm + lr * p.wpr;
-      uint32_t carry = 0;
-      for (int wi = p.wpr - 1; wi >= 0; --wi) {
-        uint32_t t = row[wi];
-        t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
-        row[wi] = (t >> 1) ^ (carry ? 0xFFFFFFFFu : 0u);
-        carry ^= (t & 1u);
-      }
-    }
+    crossings_to_bitmap(bm, p.wpr, e0, e1, p.band_edges, p.edges, p.erows, g, t, rlo, rhi, &lq);
+    suffix_xor_rows(bm, p.wpr, ch);
     __syncthreads();
     // ---- cells: stream the chunk's rows, count inside cells (fully-outside vectors are not read)
     const int16_t* base = rp.data + (rlo - rp.row0) * pitch + k0 * 8;

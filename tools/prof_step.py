@@ -12,6 +12,7 @@ from synth.dem import fill_device  # noqa: E402
 cfg = CONFIGS[sys.argv[1] if len(sys.argv) > 1 else "conus"]
 T = int(sys.argv[2]) if len(sys.argv) > 2 else cfg.tile
 steps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
+path = sys.argv[4] if len(sys.argv) > 4 else "four_step"
 P = cfg.polygons()
 pitch = (cfg.cols + 7) // 8 * 8
 r = torch.empty((cfg.rows, pitch), dtype=torch.int16, device="cuda")
@@ -19,8 +20,11 @@ fill_device(cfg.dem, cfg.cols, r.data_ptr(), 0, 0, cfg.rows, cfg.cols, pitch, to
 z = zh.ZonalHistogram(r, cfg.gt, P, cfg.nbins, tile=T, cols=cfg.cols, nodata=cfg.nodata)
 for _ in range(steps):
     z.zh_pair_tiles()
-    z.zh_tile_hist()
-    z.zh_aggregate()
-    z.zh_pip_update()
+    if path == "fused":
+        z.zh_fused_update()
+    else:
+        z.zh_tile_hist()
+        z.zh_aggregate()
+        z.zh_pip_update()
 torch.cuda.synchronize()
 print("stats", z.stats())
