@@ -5,13 +5,13 @@
 // test on the CPU "using well-established computational geometry libraries", then Thrust
 // stable_sort_by_key / stable_partition / reduce_by_key / scan to build per-polygon segments.
 // B200 design, all on the GPU:
-//   1. k_edges   — one thread per vertex: the ring edge it starts, in canonical orientation, and
+//   1. k_edges   — one CTA per polygon, one thread per vertex: the ring edge it starts, in canonical orientation, and
 //                  the exact half-open interval of centre rows it straddles (ya <= yc(r) < yb),
 //                  found with the same yc(r) expression the PIP test uses;
 //   2. k_mbb     — one CTA per polygon: vertex MBB -> covered tile rectangle (1-cell margin);
 //   3. scans     — candidate offsets and band (polygon, tile-row) bases (CUB);
-//   4. k_band_*  — per (polygon, tile row) lists of the edges whose row interval meets it (the
-//                  step-4 edge lists and the classifier's input);
+//   4. k_poly_bands — per (polygon, tile row) lists of the edges whose row interval meets it (the
+//                  step-4 edge lists and the classifier's input), counted in shared memory;
 //   5. k_mark    — a tile is INTERSECT if some edge's bounding box comes within one cell of
 //                  its cell rectangle (conservative; DESIGN.md §4 proof);
 //   6. k_classify— every other candidate tile has a uniform computed PIP status, evaluated exactly
@@ -23,15 +23,6 @@
 #include "zh_ctx.h"
 
 namespace zh {
-
-__device__ __forceinline__ int upper_bound_i32(const int32_t* a, int n, int32_t v) {
-  int lo = 0, hi = n;  // first index with a[i] > v
-  while (lo < hi) {
-    int m = (lo + hi) >> 1;
-    if (a[m] <= v) lo = m + 1; else hi = m;
-  }
-  return lo;
-}
 
 __device__ __forceinline__ int64_t upper_bound_i64(const int64_t* a, int64_t n, int64_t v) {
   int64_t lo = 0, hi = n;
@@ -66,23 +57,29 @@ __device__ __forceinline__ int2 straddle_rows(const Geo& g, double ya, double yb
   return make_int2((int)ra, (int)rb);
 }
 
-__global__ void k_edges(const int32_t* __restrict__ pro, int P, const int32_t* __restrict__ rvo, int R,
-                        const double* __restrict__ x, const double* __restrict__ y, int V, Geo g,
-                        int64_t rA, int64_t rB, int T, Edge* __restrict__ edges, int2* __restrict__ erows,
-                        int32_t* __restrict__ epoly, int32_t* __restrict__ espan) {
-  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
-    const int ring = upper_bound_i32(rvo, R + 1, v) - 1;
-    const int poly = upper_bound_i32(pro, P + 1, ring) - 1;
-    const int nxt = (v + 1 < rvo[ring + 1]) ? v + 1 : rvo[ring];
-    const double x0 = x[v], y0 = y[v], x1 = x[nxt], y1 = y[nxt];
-    Edge e;
-    if (y0 <= y1) { e.xa = x0; e.ya = y0; e.xb = x1; e.yb = y1; }
-    else          { e.xa = x1; e.ya = y1; e.xb = x0; e.yb = y0; }
-    edges[v] = e;
-    const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
-    erows[v] = rr;
-    epoly[v] = poly;
-    espan[v] = (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
+// One CTA per polygon: for every vertex v of its rings, the edge v -> next(v) (implicit closure) in
+// canonical orientation, its exact straddled row interval within the shard, its polygon and the
+// number of tile rows it spans.  (Rings are contiguous, so no search is needed.)
+__global__ void __launch_bounds__(256) k_edges(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                               const double* __restrict__ x, const double* __restrict__ y, Geo g,
+                                               int64_t rA, int64_t rB, int T, Edge* __restrict__ edges,
+                                               int2* __restrict__ erows, int32_t* __restrict__ epoly,
+                                               int32_t* __restrict__ espan) {
+  const int k = blockIdx.x;
+  for (int ring = pro[k]; ring < pro[k + 1]; ++ring) {
+    const int a = rvo[ring], b = rvo[ring + 1];
+    for (int v = a + threadIdx.x; v < b; v += blockDim.x) {
+      const int nxt = (v + 1 < b) ? v + 1 : a;
+      const double x0 = x[v], y0 = y[v], x1 = x[nxt], y1 = y[nxt];
+      Edge e;
+      if (y0 <= y1) { e.xa = x0; e.ya = y0; e.xb = x1; e.yb = y1; }
+      else          { e.xa = x1; e.ya = y1; e.xb = x0; e.yb = y0; }
+      edges[v] = e;
+      const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
+      erows[v] = rr;
+      epoly[v] = k;
+      espan[v] = (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
+    }
   }
 }
 
@@ -140,34 +137,46 @@ __global__ void __launch_bounds__(256) k_mbb(const int32_t* __restrict__ pro, co
   }
 }
 
-__global__ void k_band_count(const int2* __restrict__ erows, const int32_t* __restrict__ epoly, int V, int T,
-                             const int4* __restrict__ mbb, const int64_t* __restrict__ band_base,
-                             int32_t* __restrict__ band_cnt) {
-  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
-    const int2 rr = erows[v];
-    if (rr.x >= rr.y) continue;
-    const int k = epoly[v];
-    const int4 m = mbb[k];
-    if (m.x > m.y) continue;
-    const int64_t bb = band_base[k];
-    for (int tr = rr.x / T; tr <= (rr.y - 1) / T; ++tr) atomicAdd(&band_cnt[bb + tr - m.z], 1);
+// Band lists, one CTA per polygon: its vertices (= edges) are contiguous, and the counters of its
+// bands (one per tile row of its MBB) live in shared memory, so the heavily repeated increments of
+// consecutive edges never leave the SM.  mode 0: counts -> band_cnt; mode 1: fill band_edges from
+// band_off.  Polygons with more bands than kSmemBands use global atomics directly.
+constexpr int kSmemBands = 4096;
+__global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                                    const int2* __restrict__ erows, const int4* __restrict__ mbb,
+                                                    const int64_t* __restrict__ band_base, int T, int mode,
+                                                    int32_t* __restrict__ band_cnt, const int32_t* __restrict__ band_off,
+                                                    int32_t* __restrict__ band_edges) {
+  __shared__ int32_t sc[kSmemBands];
+  const int k = blockIdx.x;
+  const int4 m = mbb[k];
+  if (m.x > m.y) return;
+  const int nb = m.w - m.z + 1;
+  const int64_t bb = band_base[k];
+  const bool in_smem = nb <= kSmemBands;
+  int32_t* cnt = in_smem ? sc : nullptr;
+  if (in_smem) {
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) sc[i] = mode == 0 ? 0 : band_off[bb + i];
+    __syncthreads();
   }
-}
-
-__global__ void k_band_fill(const int2* __restrict__ erows, const int32_t* __restrict__ epoly, int V, int T,
-                            const int4* __restrict__ mbb, const int64_t* __restrict__ band_base,
-                            int32_t* __restrict__ band_cur, int32_t* __restrict__ band_edges) {
-  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+  const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
+  for (int v = vb + threadIdx.x; v < ve; v += blockDim.x) {
     const int2 rr = erows[v];
     if (rr.x >= rr.y) continue;
-    const int k = epoly[v];
-    const int4 m = mbb[k];
-    if (m.x > m.y) continue;
-    const int64_t bb = band_base[k];
     for (int tr = rr.x / T; tr <= (rr.y - 1) / T; ++tr) {
-      const int pos = atomicAdd(&band_cur[bb + tr - m.z], 1);
-      band_edges[pos] = v;
+      const int i = tr - m.z;
+      if (mode == 0) {
+        if (in_smem) atomicAdd(&cnt[i], 1);
+        else atomicAdd(&band_cnt[bb + i], 1);
+      } else {
+        const int pos = in_smem ? atomicAdd(&cnt[i], 1) : atomicAdd(&band_cnt[bb + i], 1);  // band_cnt = cursors
+        band_edges[pos] = v;
+      }
     }
+  }
+  if (mode == 0 && in_smem) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) band_cnt[bb + i] = sc[i];
   }
 }
 
@@ -337,10 +346,9 @@ cudaError_t launch_pairs_phase1(Ctx& c) {
   if ((e = c.d_counts.ensure(sizeof(int64_t) * 8)) != cudaSuccess) return e;
   const int64_t rA = c.rp.row0, rB = c.rp.row0 + c.rp.nrows;
   if (V > 0) {
-    k_edges<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), P, c.d_rvo.as<int32_t>(), c.R,
-                                                   c.d_x.as<double>(), c.d_y.as<double>(), V, c.geo, rA, rB,
-                                                   c.rp.T, c.d_edges.as<Edge>(), c.d_erows.as<int2>(),
-                                                   c.d_epoly.as<int32_t>(), c.d_espan.as<int32_t>());
+    k_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
+                                     c.d_y.as<double>(), c.geo, rA, rB, c.rp.T, c.d_edges.as<Edge>(),
+                                     c.d_erows.as<int2>(), c.d_epoly.as<int32_t>(), c.d_espan.as<int32_t>());
     c.launches += 1;
   }
   // one trailing zero so that the exclusive scans over P + 1 entries end with the totals
@@ -388,9 +396,9 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   // The band (polygon, tile-row) edge lists.
   cudaMemsetAsync(c.d_band_cnt.p, 0, sizeof(int32_t) * ((size_t)nb + 1), c.stream);
   if (V > 0 && nb > 0) {
-    k_band_count<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_erows.as<int2>(), c.d_epoly.as<int32_t>(), V, c.rp.T,
-                                                        c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(),
-                                                        c.d_band_cnt.as<int32_t>());
+    k_poly_bands<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
+                                          c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 0,
+                                          c.d_band_cnt.as<int32_t>(), nullptr, nullptr);
     c.launches += 1;
   }
   if (nb > 0) {
@@ -398,9 +406,10 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
       return e;
     cudaMemcpyAsync(c.d_band_cur.p, c.d_band_off.p, sizeof(int32_t) * (size_t)nb, cudaMemcpyDeviceToDevice, c.stream);
     if (V > 0) {
-      k_band_fill<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_erows.as<int2>(), c.d_epoly.as<int32_t>(), V, c.rp.T,
-                                                         c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(),
-                                                         c.d_band_cur.as<int32_t>(), c.d_band_edges.as<int32_t>());
+      k_poly_bands<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
+                                            c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 1,
+                                            c.d_band_cur.as<int32_t>(), c.d_band_off.as<int32_t>(),
+                                            c.d_band_edges.as<int32_t>());
       c.launches += 1;
     }
   }
