@@ -226,9 +226,17 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # ZH_BENCH_SHARED_GPU=1: every rank on cuda:0 with gloo — exercises the multi-rank code path on a
+    # one-GPU box (numbers are not a scaling measurement then).  Default: one GPU per rank, NCCL.
+    shared = os.environ.get("ZH_BENCH_SHARED_GPU", "0") == "1"
+    if shared:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
     def log(*a):
         if args.verbose and rank == 0:
@@ -388,7 +396,8 @@ def main():
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
                 "data": "synthetic (fractal int16 DEM + jagged Voronoi counties, seeded)",
-                "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert, parallelism=f"tile-row shards x{world}",
+                "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert,
+                               parallelism=f"tile-row shards x{world}" + (" (shared GPU, gloo)" if shared else ""),
                                l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA"),
                 "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
                 "clocks": clocks, "path": path, "steps_detail": steps_detail, "other_path": other,

@@ -1,0 +1,91 @@
+"""The multi-GPU path on one GPU: world_size 2 processes (torch.distributed, gloo over the same
+cuda:0 — there is one GPU in this environment), each holding a tile-row strip of the tiny and
+state rasters in HBM, running libzh on its strip (both paths), and all-reducing the int64 view of
+the uint64 histograms.  The reduced result must equal the oracle bit for bit."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, cfg_name, q):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangw14_b200 import zh
+    from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms, shard_rows
+    from synth.configs import CONFIGS
+    from synth.dem import fill_device
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        cfg = CONFIGS[cfg_name]
+        P = cfg.polygons()
+        r0, r1 = shard_rows(cfg.rows, cfg.tile, world, rank)
+        pitch = (cfg.cols + 7) // 8 * 8
+        t = torch.empty((max(r1 - r0, 1), pitch), dtype=torch.int16, device="cuda")
+        fill_device(cfg.dem, cfg.cols, t.data_ptr(), r0, 0, r1 - r0, cfg.cols, pitch,
+                    torch.cuda.current_stream().cuda_stream)
+        res = []
+        for fused in (False, True):
+            out = torch.zeros((P.n_poly, cfg.nbins), dtype=torch.int64, device="cuda")
+            with zh.ZonalHistogram(t[:r1 - r0], cfg.gt, P, cfg.nbins, tile=cfg.tile, rows=cfg.rows, cols=cfg.cols,
+                                   row0=r0, nodata=cfg.nodata, fused=fused) as z:
+                z.set_output(out)
+                z.zh_run(None)
+            reduce_histograms(out)
+            res.append(out.cpu().numpy().view(np.uint64).copy())
+        q.put((rank, res[0], res[1]))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("cfg_name", ["tiny", "state"])
+def test_two_ranks_reduce_to_oracle(cuda_device, cfg_name):
+    import torch.multiprocessing as mp
+
+    import oracle
+    from synth.configs import CONFIGS
+    from synth.dem import fill_host
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg_name, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = [q.get(timeout=600) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    cfg = CONFIGS[cfg_name]
+    P = cfg.polygons()
+    bins = oracle.make_bins(cfg.nbins, nodata=cfg.nodata)
+    if cfg_name == "tiny":
+        R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
+        want = oracle.o1(R, cfg.gt, P, bins)
+        rows = range(P.n_poly)
+    else:  # state: sampled polygons, each from its own raster window
+        rows = [0, P.n_poly // 2, P.n_poly - 1]
+        want = np.zeros((P.n_poly, cfg.nbins), np.uint64)
+        for k in rows:
+            r0, r1, c0, c1 = oracle.polygon_window(P, k, cfg.gt, cfg.rows, cfg.cols)
+            win = fill_host(cfg.dem, cfg.cols, r0, c0, r1 - r0, c1 - c0)
+            want[k] = oracle.o1(win, cfg.gt, P.subset([k]), bins, row0=r0, col0=c0)[0]
+    for rank, four, fused in got:
+        assert (four == fused).all()
+        for k in rows:
+            assert (fused[k] == want[k]).all(), (rank, k)
