@@ -18,9 +18,9 @@ pitch = (cfg.cols + 7) // 8 * 8
 r = torch.empty((cfg.rows, pitch), dtype=torch.int16, device="cuda")
 fill_device(cfg.dem, cfg.cols, r.data_ptr(), 0, 0, cfg.rows, cfg.cols, pitch, torch.cuda.current_stream().cuda_stream)
 z = zh.ZonalHistogram(r, cfg.gt, P, cfg.nbins, tile=T, cols=cfg.cols, nodata=cfg.nodata)
-for _ in range(steps):
+for i in range(steps):
     z.zh_pair_tiles()
-    if path == "fused":
+    if path == "fused" or (path == "four_fused" and i % 2 == 1):
         z.zh_fused_update()
     else:
         z.zh_tile_hist()
