@@ -9,7 +9,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libzh.so")
 SOURCES = ["zh_api.cu", "k_tile_hist.cu", "k_pairs.cu", "k_aggregate.cu", "k_pip.cu", "k_fused.cu"]
-HEADERS = ["zh_internal.cuh", "zh_ctx.h", "zh_tilehist.cuh", "zh_parity.cuh"]
+HEADERS = ["zh_internal.cuh", "zh_ctx.h", "zh_tilehist.cuh", "zh_parity.cuh", "zh_pip.cuh"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-O3"]

@@ -14,6 +14,7 @@
 #include <cub/device/device_scan.cuh>
 
 #include "zh_ctx.h"
+#include "zh_pip.cuh"
 #include "zh_tilehist.cuh"
 
 namespace zh {
@@ -103,35 +104,48 @@ __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, cons
                                                   (unsigned long long)cells);
 }
 
+struct PureP {
+  RasterP rp;
+  BinP bp;
+  FastBins fb;
+  const int32_t* pure_tiles;
+  const int64_t* counts;
+  const uint64_t* pure_off;
+  const uint32_t* pure_cnt;
+  const int32_t* pure_poly;
+  void* out;
+};
+
+// One pure tile: the step-1 shared histogram, added into each inside polygon's row.
 template <int kMode, bool kU64>
-__global__ void __launch_bounds__(512, 3) k_fused_pure(RasterP rp, BinP bp, FastBins fb,
-                                                       const int32_t* __restrict__ pure_tiles,
-                                                       const int64_t* __restrict__ counts,
-                                                       const uint64_t* __restrict__ pure_off,
-                                                       const uint32_t* __restrict__ pure_cnt,
-                                                       const int32_t* __restrict__ pure_poly, void* __restrict__ out) {
-  if ((int64_t)blockIdx.x >= counts[0]) return;
-  extern __shared__ __align__(16) uint32_t sh[];
-  const int HW = hist_words(bp.nbins);
-  const int tile = pure_tiles[blockIdx.x];
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+__device__ __forceinline__ void pure_tile_body(const PureP& f, int64_t idx, uint32_t* __restrict__ sh) {
+  const int HW = hist_words(f.bp.nbins);
+  const int tile = f.pure_tiles[idx];
+  const int trl = tile / f.rp.TC, tc = tile - trl * f.rp.TC;
   for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
     *reinterpret_cast<uint4*>(&sh[i]) = make_uint4(0, 0, 0, 0);
   __syncthreads();
-  tile_histogram<kMode>(sh, rp, bp, fb, trl, tc);
+  tile_histogram<kMode>(sh, f.rp, f.bp, f.fb, trl, tc);
   __syncthreads();
-  const uint32_t beg = (uint32_t)(pure_off[tile] & 0xFFFFFFFFull), cnt = pure_cnt[tile];
-  const int nbins = bp.nbins;
+  const uint32_t beg = (uint32_t)(f.pure_off[tile] & 0xFFFFFFFFull), cnt = f.pure_cnt[tile];
+  const int nbins = f.bp.nbins;
   for (uint32_t j = 0; j < cnt; ++j) {
-    const int64_t row = (int64_t)pure_poly[beg + j] * nbins;
+    const int64_t row = (int64_t)f.pure_poly[beg + j] * nbins;
     for (int b = threadIdx.x; b < nbins; b += blockDim.x) {
       const uint32_t v = sh[kOff + b];
       if (v) {
-        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(out) + row + b, (unsigned long long)v);
-        else atomicAdd(reinterpret_cast<uint32_t*>(out) + row + b, v);
+        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(f.out) + row + b, (unsigned long long)v);
+        else atomicAdd(reinterpret_cast<uint32_t*>(f.out) + row + b, v);
       }
     }
   }
+}
+
+template <int kMode, bool kU64>
+__global__ void __launch_bounds__(512, 3) k_fused_pure(PureP f) {
+  if ((int64_t)blockIdx.x >= f.counts[0]) return;
+  extern __shared__ __align__(16) uint32_t sh[];
+  pure_tile_body<kMode, kU64>(f, blockIdx.x, sh);
 }
 
 static int grid_for(int64_t n, int threads) {
@@ -152,13 +166,25 @@ static cudaError_t excl_scan(Ctx& c, const T* in, T* out, int64_t n) {
   return cub::DeviceScan::ExclusiveSum(c.d_cub.p, have, in, out, (int)n, c.stream);
 }
 
+static PureP pure_params(Ctx& c) {
+  PureP f;
+  f.rp = c.rp;
+  f.bp = c.bp;
+  f.fb = make_fast_bins(c.bp);
+  f.pure_tiles = c.d_pure_tiles.as<int32_t>();
+  f.counts = c.d_fcounts.as<int64_t>();
+  f.pure_off = c.d_pure_off.as<uint64_t>();
+  f.pure_cnt = c.d_pure_cnt.as<uint32_t>();
+  f.pure_poly = c.d_pure_poly.as<int32_t>();
+  f.out = c.d_out;
+  return f;
+}
+
 template <int kMode, bool kU64>
 static void launch_pure(Ctx& c, size_t smem, unsigned grid) {
   auto k = k_fused_pure<kMode, kU64>;
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k<<<grid, 512, smem, c.stream>>>(c.rp, c.bp, make_fast_bins(c.bp), c.d_pure_tiles.as<int32_t>(),
-                                   c.d_fcounts.as<int64_t>(), c.d_pure_off.as<uint64_t>(),
-                                   c.d_pure_cnt.as<uint32_t>(), c.d_pure_poly.as<int32_t>(), c.d_out);
+  k<<<grid, 512, smem, c.stream>>>(pure_params(c));
 }
 
 cudaError_t launch_fused(Ctx& c) {
@@ -217,13 +243,14 @@ cudaError_t launch_fused(Ctx& c) {
                                                           c.rp, c.d_pip.as<int2>(), c.d_fcounts.as<int64_t>());
   c.launches += 1;
 
+  const int mode = fast_bins_ok(c.bp) ? (make_fast_bins(c.bp).bias ? 4 : (c.bp.use_nodata ? 3 : 2))
+                                      : (c.bp.width == 1 ? 0 : 1);
+  // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
   // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
   if (c.timing) cudaEventRecord(c.ev[10], c.stream);
   if (NI > 0) {
     const size_t smem = (size_t)hist_words(c.bp.nbins) * 4;
     const unsigned grid = (unsigned)NI;
-    const int mode = fast_bins_ok(c.bp) ? (make_fast_bins(c.bp).bias ? 4 : (c.bp.use_nodata ? 3 : 2))
-                                        : (c.bp.width == 1 ? 0 : 1);
     if (c.out_u64) {
       switch (mode) {
         case 0: launch_pure<0, true>(c, smem, grid); break;
