@@ -165,6 +165,18 @@ zh_status zh_fused_update(zh_ctx ctx);
  * out_u64, row-major [n_poly][nbins]) to host_out (may be NULL to skip the copy).  Syncs. */
 zh_status zh_run(zh_ctx ctx, void* host_out);
 
+/* Zonal statistics from the histograms (the classic per-zone min, max, average,
+ * count and standard deviation of PAPER.md:10 §I ¶1), exact integers in units of bin indices b
+ * (value of bin b = lo + b * width).  Per polygon ZH_NSTATS int64:
+ *   [0] count  [1] min_bin  [2] max_bin  [3] lower-median bin  (bins -1 for an empty polygon)
+ *   [4] sum of b  [5],[6] sum of b^2 as (low, high) 64-bit words of a 128-bit integer
+ *   [7] number of non-zero bins
+ * Needs a completed histogram since the last zh_pair_tiles (zh_run, steps 3+4, or the fused
+ * update).  host_stats (n_poly * ZH_NSTATS, may be NULL) receives a copy (syncs); *dptr (may be
+ * NULL) a BORROWED device pointer. */
+#define ZH_NSTATS 8
+zh_status zh_zonal_stats(zh_ctx ctx, int64_t* host_stats, int64_t** dptr);
+
 /* BORROWED device pointer to the output ([n_poly][nbins], uint64 or uint32) — e.g. for an
  * NCCL reduce across shards.  *n = n_poly * nbins elements. */
 zh_status zh_output_device(zh_ctx ctx, void** dptr, int64_t* n);

@@ -155,3 +155,30 @@ def polygon_window(P, k: int, gt, rows: int, cols: int, margin: int = 2):
     r0 = max(0, int(np.floor(rr.min())) - margin)
     r1 = min(rows, int(np.ceil(rr.max())) + margin)
     return r0, max(r0, r1), c0, max(c0, c1)
+
+
+def zonal_stats(H) -> np.ndarray:
+    """Zonal statistics of each histogram row, the plain definition in exact Python integers
+    (min/max/average/count/std of PAPER.md:10 §I ¶1), in units of bin indices:
+    [count, min_bin, max_bin, lower-median bin, sum b, sum b^2 low word, sum b^2 high word,
+    non-zero bins]; bins are -1 for an empty row."""
+    H = np.asarray(H)
+    out = np.zeros((H.shape[0], 8), dtype=np.int64)
+    for k in range(H.shape[0]):
+        row = [int(v) for v in H[k]]
+        n = sum(row)
+        nzb = [b for b, v in enumerate(row) if v]
+        s1 = sum(b * v for b, v in enumerate(row))
+        s2 = sum(b * b * v for b, v in enumerate(row))
+        med = -1
+        if n:
+            target, run = (n + 1) // 2, 0
+            for b, v in enumerate(row):
+                run += v
+                if run >= target:
+                    med = b
+                    break
+        lo64 = s2 & ((1 << 64) - 1)
+        out[k] = [n, nzb[0] if nzb else -1, nzb[-1] if nzb else -1, med, s1,
+                  lo64 - (1 << 64) if lo64 >= (1 << 63) else lo64, s2 >> 64, len(nzb)]
+    return out

@@ -202,7 +202,7 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
-                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_fcounts};
+                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_fcounts, &c->d_stats};
   for (auto* b : bufs) b->release();
   for (int i = 0; i < 13; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
@@ -217,7 +217,7 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
-                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_fcounts};
+                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_fcounts, &c.d_stats};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;
@@ -343,6 +343,23 @@ extern "C" zh_status zh_run(zh_ctx h, void* host_out) {
     ZH_CU(cudaMemcpyAsync(host_out, c->d_out, out_bytes, cudaMemcpyDeviceToHost, c->stream), "zh_run (D2H)");
   }
   ZH_CU(cudaStreamSynchronize(c->stream), "zh_run (sync)");
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_zonal_stats(zh_ctx h, int64_t* host_stats, int64_t** dptr) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (!c->have_pairs || !(c->fused_done || c->step4_done))
+    return fail(ZH_ERR_STATE, "zh_zonal_stats needs a completed histogram (zh_run or steps 2 + 3/4 or fused)");
+  ZH_CU(c->d_stats.ensure((size_t)(c->P > 0 ? c->P : 1) * ZH_NSTATS * sizeof(int64_t)), "zh_zonal_stats");
+  ZH_CU(zh::launch_zonal_stats(*c, c->d_stats.as<int64_t>()), "zh_zonal_stats");
+  if (dptr) *dptr = c->d_stats.as<int64_t>();
+  if (host_stats && c->P > 0) {
+    ZH_CU(cudaMemcpyAsync(host_stats, c->d_stats.p, (size_t)c->P * ZH_NSTATS * sizeof(int64_t),
+                          cudaMemcpyDeviceToHost, c->stream),
+          "zh_zonal_stats (D2H)");
+    ZH_CU(cudaStreamSynchronize(c->stream), "zh_zonal_stats");
+  }
   return ZH_OK;
 }
 

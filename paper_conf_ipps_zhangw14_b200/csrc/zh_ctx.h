@@ -55,6 +55,7 @@ struct Ctx {
   // fused path lists (k_fused.cu)
   DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,
       d_pip, d_fcounts;
+  DBuf d_stats;  // zonal statistics [P][8] (k_stats.cu)
   int64_t n_cand = 0, n_bands = 0, n_band_entries = 0, n_inside = 0, n_isect = 0;
   // step 1 product and output
   DBuf d_tile_hist;
@@ -81,6 +82,7 @@ cudaError_t launch_aggregate(Ctx& c);
 cudaError_t launch_pip(Ctx& c);
 cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
 cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
+cudaError_t launch_zonal_stats(Ctx& c, int64_t* dstats);  // k_stats.cu
 
 size_t device_bytes(const Ctx& c);
 

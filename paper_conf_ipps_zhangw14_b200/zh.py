@@ -60,7 +60,7 @@ class zh_stats(ctypes.Structure):
 
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",
-           "zh_fused_update",
+           "zh_fused_update", "zh_zonal_stats",
            "zh_run", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
            "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy"]
 
@@ -81,6 +81,7 @@ def _load():
         "zh_aggregate": (st, [vp]),
         "zh_pip_update": (st, [vp]),
         "zh_fused_update": (st, [vp]),
+        "zh_zonal_stats": (st, [vp, vp, vp]),
         "zh_run": (st, [vp, vp]),
         "zh_output_device": (st, [vp, ctypes.POINTER(vp), ctypes.POINTER(i64)]),
         "zh_set_output": (st, [vp, vp]),
@@ -223,6 +224,29 @@ class ZonalHistogram:
     def run(self) -> np.ndarray:
         out = np.empty((self.n_poly, self.nbins), dtype=np.uint64 if self.out_u64 else np.uint32)
         return self.zh_run(out)
+
+    def zh_zonal_stats(self) -> np.ndarray:
+        """Raw exact statistics [n_poly, 8] int64 (see zh.h: count, min/max/median bin, sum b,
+        sum b^2 low/high words, non-zero bins)."""
+        out = np.zeros((self.n_poly, 8), dtype=np.int64)
+        _check(LIB.zh_zonal_stats(self.h, out.ctypes.data if self.n_poly else None, None))
+        return out
+
+    def zonal_stats(self, lo: int = 0, width: int = 1) -> dict:
+        """count, min, max, median, mean, std per polygon in value units (value of bin b =
+        lo + b * width), derived from zh_zonal_stats' exact integers."""
+        raw = self.zh_zonal_stats()
+        n = raw[:, 0].astype(np.float64)
+        s = raw[:, 4].astype(np.float64)
+        sq = raw[:, 5].view(np.uint64).astype(np.float64) + raw[:, 6].astype(np.float64) * 2.0 ** 64
+        with np.errstate(invalid="ignore", divide="ignore"):
+            mean_b = s / n
+            var_b = np.maximum(sq / n - mean_b * mean_b, 0.0)
+        empty = raw[:, 0] == 0
+        val = lambda b: np.where(empty, np.nan, lo + b * width)
+        return {"count": raw[:, 0], "min": val(raw[:, 1]), "max": val(raw[:, 2]), "median": val(raw[:, 3]),
+                "mean": np.where(empty, np.nan, lo + mean_b * width),
+                "std": np.where(empty, np.nan, np.sqrt(var_b) * width), "nonzero_bins": raw[:, 7]}
 
     def output_device(self):
         """The output as a torch CUDA tensor view (int64 for u64, int32 for u32 — same bits)."""

@@ -262,3 +262,25 @@ def test_overlapping_polygons_and_linear_pattern(cuda_device):
     t = device_raster(spec, rows, cols)
     for tile in (32, 64, 256):
         assert (gpu_hist(t, gt, P, 4096, tile, cols, lo=-7) == H).all()
+
+
+@pytest.mark.parametrize("out_u64", [True, False])
+def test_zonal_stats_match_oracle(tiny, cuda_device, out_u64):
+    """zh_zonal_stats (exact integers from the device histogram) == the oracle's
+    statistics of the oracle histogram; clamped default bins and an unclamped mapping."""
+    cfg, P, R, H = tiny
+    zh = _zh()
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    for lo, nb in ((0, cfg.nbins), (-400, 1200)):
+        Hb = H if lo == 0 else oracle.o1(R, cfg.gt, P, oracle.make_bins(nb, lo=lo, nodata=cfg.nodata))
+        want = oracle.zonal_stats(Hb)
+        for fused in (False, True):
+            with zh.ZonalHistogram(t, cfg.gt, P, nb, lo=lo, tile=cfg.tile, cols=cfg.cols, nodata=cfg.nodata,
+                                   out_u64=out_u64, fused=fused) as z:
+                z.run()
+                got = z.zh_zonal_stats()
+                derived = z.zonal_stats(lo=lo)
+            assert (got == want).all()
+            nz = want[:, 0] > 0
+            assert np.allclose(derived["min"][nz], lo + want[nz, 1])
+            assert (derived["count"] == want[:, 0]).all()

@@ -225,3 +225,31 @@ def test_degenerate_inputs():
         assert H[0:4].sum() == 0 and H[7].sum() == 0
         assert (H[4] == H[5]).all() and (H[4] == H[6]).all() and (H[4] == H[8]).all()
         assert H[4].sum() > 0
+
+
+def test_zonal_stats_from_histogram_match_cells():
+    """oracle.zonal_stats (from the oracle histogram) == the same statistics computed straight
+    from the cell values inside each polygon (oracle membership), with no clamping in play."""
+    cfg = TINY
+    P = cfg.polygons()
+    R = fill_host(cfg.dem, cfg.cols, 0, 0, 256, 384)  # a window; polygons cover it partially
+    gt = (0.0, 1.0, 0.0, 1024.0, 0.0, -1.0)
+    lo, nb = -400, 1200  # every DEM value of the window has its own bin
+    H = oracle.o1(R, gt, P, oracle.make_bins(nb, lo=lo, nodata=-32768))
+    st = oracle.zonal_stats(H)
+    rr, cc = np.meshgrid(np.arange(256), np.arange(384), indexing="ij")
+    mem = oracle.membership(rr.ravel(), cc.ravel(), gt, P)
+    vals = R.ravel().astype(np.int64)
+    for k in range(P.n_poly):
+        sel = (mem[:, k] == 1) & (vals != -32768)
+        b = vals[sel] - lo
+        assert st[k, 0] == b.size
+        if b.size == 0:
+            assert st[k, 1] == st[k, 2] == st[k, 3] == -1
+            continue
+        assert st[k, 1] == b.min() and st[k, 2] == b.max()
+        assert st[k, 3] == np.sort(b)[(b.size + 1) // 2 - 1]
+        assert st[k, 4] == b.sum()
+        s2 = int((b * b).sum())
+        assert st[k, 5] == np.int64(np.uint64(s2 & ((1 << 64) - 1)).view(np.int64)) and st[k, 6] == s2 >> 64
+        assert st[k, 7] == np.unique(b).size
