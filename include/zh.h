@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 2
+#define ZH_ABI_VERSION 3
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -66,7 +66,8 @@ typedef enum {
  * on_host = 1: `data` is HOST memory (borrowed; pin it for full PCIe speed); the context owns a
  *   device copy and every zh_run / zh_upload_raster copies the shard host->device first.
  * Geotransform (GDAL): x = gt[0] + col*gt[1] + row*gt[2], y = gt[3] + col*gt[4] + row*gt[5];
- *   the cell (r, c) has centre x = gt[0] + (c + 0.5)*gt[1], y = gt[3] + (r + 0.5)*gt[5].
+ *   the cell (r, c) has centre x = gt[0] + (c + 0.5)*gt[1], y = gt[3] + (r + 0.5)*gt[5]
+ *   (with options.rep_custom: (c + rep_x), (r + rep_y) instead of the 0.5s).
  *   gt[2] and gt[4] must be 0 (north-up; rotated -> UNSUPPORTED); gt[1], gt[5] nonzero, finite.
  * Sharding (multi-GPU): a rank holds rows [row0, row0 + nrows) of an M x N raster; row0 must be
  *   a multiple of the tile size so that shards consist of whole tile rows. */
@@ -117,6 +118,12 @@ typedef struct {
                           work; a validation mode — the result must not change)                  */
   int32_t fused;       /* 1: zh_run uses zh_fused_update instead of steps 1, 3, 4               */
   void* stream;        /* cudaStream_t                                                          */
+  int32_t rep_custom;  /* 0: the cell CENTRE is the representative point (§III.D);
+                          1: the point (c + rep_x, r + rep_y) in cell units, rep_x, rep_y in
+                          [0, 1] — e.g. (0, 0) the cell corner at the origin of the cell
+                          (the alternatives of PAPER.md:18)                   */
+  int32_t reserved;
+  double rep_x, rep_y;
 } zh_options;
 
 typedef struct {

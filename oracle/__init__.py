@@ -75,6 +75,13 @@ def _c64(a, dt):
     return np.ascontiguousarray(a, dtype=dt)
 
 
+def _gt8(gt, rep=None):
+    """gt (6 GDAL coefficients) + the representative point offsets (default: the cell centre)."""
+    g = [float(v) for v in gt][:6]
+    r = (0.5, 0.5) if rep is None else (float(rep[0]), float(rep[1]))
+    return np.array(g + list(r), dtype=np.float64)
+
+
 def _poly_args(P):
     pro = _c64(P.poly_ring_off, np.int64)
     rvo = _c64(P.ring_vert_off, np.int64)
@@ -91,8 +98,8 @@ def bin_of(v: int, bins: Bins) -> int:
     return int(_L().zho_bin(int(v), ctypes.byref(bins)))
 
 
-def centre(gt, r: int, c: int):
-    g = _c64(gt, np.float64)
+def centre(gt, r: int, c: int, rep=None):
+    g = _gt8(gt, rep)
     xc, yc = ctypes.c_double(), ctypes.c_double()
     _L().zho_centre(g.ctypes.data, r, c, ctypes.byref(xc), ctypes.byref(yc))
     return xc.value, yc.value
@@ -104,12 +111,12 @@ def crossings(P, k: int, xc: float, yc: float) -> int:
                                   x.ctypes.data, y.ctypes.data))
 
 
-def _hist(fn, win, row0, col0, gt, P, bins, nthreads, extra):
+def _hist(fn, win, row0, col0, gt, P, bins, nthreads, extra, rep=None):
     win = np.asarray(win)
     assert win.dtype == np.int16 and win.ndim == 2 and win.strides[1] == 2
     nrows, ncols = win.shape
     pitch = win.strides[0] // 2
-    g = _c64(gt, np.float64)
+    g = _gt8(gt, rep)
     pro, rvo, x, y = _poly_args(P)
     out = np.zeros((P.n_poly, bins.nbins), dtype=np.uint64)
     fn(win.ctypes.data, int(row0), int(col0), nrows, ncols, pitch, g.ctypes.data, P.n_poly,
@@ -118,21 +125,22 @@ def _hist(fn, win, row0, col0, gt, P, bins, nthreads, extra):
     return out
 
 
-def o0(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, prefilter: bool = False, nthreads=None):
-    """O0: the definition (every cell x polygon x edge).  Returns uint64 [n_poly, nbins]."""
-    return _hist(_L().zho_o0, win, row0, col0, gt, P, bins, nthreads, (int(prefilter),))
+def o0(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, prefilter: bool = False, nthreads=None, rep=None):
+    """O0: the definition (every cell x polygon x edge).  Returns uint64 [n_poly, nbins].
+    rep: representative point offsets in the cell (default (0.5, 0.5), the centre)."""
+    return _hist(_L().zho_o0, win, row0, col0, gt, P, bins, nthreads, (int(prefilter),), rep)
 
 
-def o1(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, nthreads=None):
+def o1(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, nthreads=None, rep=None):
     """O1: row-hoisted intercepts, identical comparisons to O0.  Returns uint64 [n_poly, nbins]."""
-    return _hist(_L().zho_o1, win, row0, col0, gt, P, bins, nthreads, ())
+    return _hist(_L().zho_o1, win, row0, col0, gt, P, bins, nthreads, (), rep)
 
 
-def membership(rows, cols, gt, P, nthreads=None) -> np.ndarray:
+def membership(rows, cols, gt, P, nthreads=None, rep=None) -> np.ndarray:
     """inside[q, k] in {0,1} for the cells (rows[q], cols[q])."""
     rows = _c64(rows, np.int64)
     cols = _c64(cols, np.int64)
-    g = _c64(gt, np.float64)
+    g = _gt8(gt, rep)
     pro, rvo, x, y = _poly_args(P)
     out = np.zeros((rows.shape[0], P.n_poly), dtype=np.uint8)
     _L().zho_membership(rows.ctypes.data, cols.ctypes.data, rows.shape[0], g.ctypes.data, P.n_poly,

@@ -61,10 +61,12 @@ int zho_bin(int32_t v, const zho_bins* b) {
   return q;
 }
 
-/* Cell centre (GDAL convention, north-up: gt2 = gt4 = 0). */
+/* Cell centre (GDAL convention, north-up: gt2 = gt4 = 0).  gt has 8 entries: gt[6], gt[7] are the
+ * representative point's offsets inside the cell in cell units — 0.5, 0.5 for the centre the paper
+ * chooses (§III.D); other points are its alternatives (e.g. 0, 0: a corner). */
 void zho_centre(const double* gt, int64_t r, int64_t c, double* xc, double* yc) {
-  double cc = (double)c + 0.5;
-  double rr = (double)r + 0.5;
+  double cc = (double)c + gt[6];
+  double rr = (double)r + gt[7];
   double tx = cc * gt[1];
   double ty = rr * gt[5];
   *xc = gt[0] + tx;
@@ -216,8 +218,8 @@ void zho_o1(const int16_t* win, int64_t row0, int64_t col0, int64_t nrows, int64
          * cell exactly; when n is odd (cannot happen for closed rings) visit the whole row. */
         int64_t jlo = 0, jhi = ncols; /* window-relative, half-open */
         if ((n & 1) == 0) {
-          double clo = (xs[0] - gt[0]) / gt[1] - 0.5;
-          double chi = (xs[n - 1] - gt[0]) / gt[1] - 0.5;
+          double clo = (xs[0] - gt[0]) / gt[1] - gt[6];
+          double chi = (xs[n - 1] - gt[0]) / gt[1] - gt[6];
           if (clo > chi) { double t = clo; clo = chi; chi = t; }
           double a0 = floor(clo) - 2 - (double)col0, a1 = ceil(chi) + 3 - (double)col0;
           if (a0 > (double)jlo) jlo = a0 > (double)ncols ? ncols : (int64_t)a0;

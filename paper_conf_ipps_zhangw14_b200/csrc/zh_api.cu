@@ -52,6 +52,8 @@ static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bin
   if (r->row0 < 0 || r->nrows < 0 || r->row0 + r->nrows > r->rows)
     return fail(ZH_ERR_INVALID_ARG, "shard rows [row0, row0+nrows) outside the raster");
   if (o->tile < 1) return fail(ZH_ERR_INVALID_ARG, "tile must be >= 1");
+  if (o->rep_custom && !(o->rep_x >= 0.0 && o->rep_x <= 1.0 && o->rep_y >= 0.0 && o->rep_y <= 1.0))
+    return fail(ZH_ERR_INVALID_ARG, "representative point offsets must lie in [0, 1]");
   if (r->row0 % o->tile != 0) return fail(ZH_ERR_INVALID_ARG, "row0 must be a multiple of the tile size");
   for (int i = 0; i < 6; ++i)
     if (!isfinite(r->gt[i])) return fail(ZH_ERR_INVALID_ARG, "geotransform must be finite");
@@ -136,7 +138,8 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   c->rp.TC = (int32_t)TC;
   c->rp.tr0 = (int32_t)tr0;
   c->rp.TRn = (int32_t)TRn;
-  c->geo = zh::Geo{r->gt[0], r->gt[1], r->gt[3], r->gt[5]};
+  c->geo = zh::Geo{r->gt[0], r->gt[1], r->gt[3], r->gt[5], o->rep_custom ? o->rep_x : 0.5,
+                   o->rep_custom ? o->rep_y : 0.5};
   c->on_host = r->on_host != 0;
   c->host_data = r->on_host ? r->data : nullptr;
   c->bp = zh::BinP{b->lo, b->width, b->nbins, b->use_nodata ? 1 : 0, b->nodata, b->oor_drop ? 1 : 0};

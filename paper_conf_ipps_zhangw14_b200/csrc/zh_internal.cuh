@@ -13,15 +13,19 @@ namespace zh {
 // Geometry: cell centres and Franklin's intercept, each operation an explicit IEEE binary64
 // round-to-nearest op (__d*_rn) so that nvcc cannot contract them into FMAs (DESIGN.md §3 R7).
 // ----------------------------------------------------------------------------------------------
+// (ox, oy): the representative point inside the cell, in cell units — (0.5, 0.5) is the centre the
+// paper chooses (§III.D); other points (corners, ...) are the alternatives it mentions
+// (SURVEY.md §8f-3).  The names below say "centre" for the general representative point.
 struct Geo {
   double gt0, gt1, gt3, gt5;
+  double ox, oy;
 };
 
 __device__ __forceinline__ double col_centre(const Geo& g, int64_t c) {
-  return __dadd_rn(g.gt0, __dmul_rn(__dadd_rn((double)c, 0.5), g.gt1));
+  return __dadd_rn(g.gt0, __dmul_rn(__dadd_rn((double)c, g.ox), g.gt1));
 }
 __device__ __forceinline__ double row_centre(const Geo& g, int64_t r) {
-  return __dadd_rn(g.gt3, __dmul_rn(__dadd_rn((double)r, 0.5), g.gt5));
+  return __dadd_rn(g.gt3, __dmul_rn(__dadd_rn((double)r, g.oy), g.gt5));
 }
 
 // Canonical edge (ya <= yb), Fig. 5 predicate in lower-endpoint-first orientation (R8).

@@ -45,7 +45,7 @@ __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr,
   const int w = t.w;
   const double yc = row_centre(g, r);
   const double xi = intercept(e, yc);
-  const double est = (xi - g.gt0) / g.gt1 - 0.5 - (double)t.c0;
+  const double est = (xi - g.gt0) / g.gt1 - g.ox - (double)t.c0;
   int64_t ei;
   if (!(est > 0.0)) ei = 0;
   else if (est > (double)w) ei = w;

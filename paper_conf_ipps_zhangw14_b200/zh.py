@@ -49,7 +49,8 @@ class zh_bins(ctypes.Structure):
 
 class zh_options(ctypes.Structure):
     _fields_ = [("tile", ctypes.c_int32), ("out_u64", ctypes.c_int32), ("force_isect", ctypes.c_int32),
-                ("fused", ctypes.c_int32), ("stream", ctypes.c_void_p)]
+                ("fused", ctypes.c_int32), ("stream", ctypes.c_void_p), ("rep_custom", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("rep_x", ctypes.c_double), ("rep_y", ctypes.c_double)]
 
 
 class zh_stats(ctypes.Structure):
@@ -140,12 +141,13 @@ class ZonalHistogram:
     host numpy/torch int16 array (on_host; pinned memory recommended).  Its first row is global
     row `row0` of a raster with `rows` rows (default: a single shard holding the whole raster).
     polygons: any object with poly_ring_off, ring_vert_off, x, y arrays (synth.polygons.Polygons).
+    rep: None for cell centres, or (ox, oy) in [0, 1]^2 — the representative point (c+ox, r+oy).
     """
 
     def __init__(self, raster, gt, polygons, nbins: int, lo: int = 0, width: int = 1, nodata=None,
                  oor_drop: bool = False, tile: int = 256, out_u64: bool = True, force_isect: bool = False,
                  row0: int = 0, rows: int | None = None, cols: int | None = None, stream=None,
-                 fused: bool = True):
+                 fused: bool = True, rep=None):
         self._keep = []
         on_host, ptr, nrows, ncols_buf, pitch = self._raster_ptr(raster)
         ncols = cols if cols is not None else ncols_buf
@@ -166,7 +168,9 @@ class ZonalHistogram:
                         x.ctypes.data, y.ctypes.data)
         b = zh_bins(lo, width, nbins, 0 if nodata is None else 1, 0 if nodata is None else int(nodata), int(oor_drop))
         self.stream = _stream_handle(stream)
-        o = zh_options(tile, int(out_u64), int(force_isect), int(fused), self.stream)
+        o = zh_options(tile, int(out_u64), int(force_isect), int(fused), self.stream,
+                       0 if rep is None else 1, 0, 0.5 if rep is None else float(rep[0]),
+                       0.5 if rep is None else float(rep[1]))
         h = ctypes.c_void_p()
         _check(LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)))
         self.h = h

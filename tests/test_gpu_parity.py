@@ -284,3 +284,19 @@ def test_zonal_stats_match_oracle(tiny, cuda_device, out_u64):
             nz = want[:, 0] > 0
             assert np.allclose(derived["min"][nz], lo + want[nz, 1])
             assert (derived["count"] == want[:, 0]).all()
+
+
+@pytest.mark.parametrize("rep", [(0.0, 0.0), (0.0, 1.0), (1.0, 1.0), (0.25, 0.75)])
+def test_representative_points(tiny, cuda_device, rep):
+    """cell corners / arbitrary points of the cell instead of the centre."""
+    cfg, P, R, _ = tiny
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata), rep=rep)
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    for tile in (64, 128):
+        assert (gpu_hist(t, cfg.gt, P, cfg.nbins, tile, cfg.cols, nodata=cfg.nodata, rep=rep) == H).all()
+    lon = TINY_LONLAT
+    P2 = lon.polygons()
+    R2 = fill_host(lon.dem, lon.cols, 0, 0, lon.rows, lon.cols)
+    H2 = oracle.o1(R2, lon.gt, P2, oracle.make_bins(lon.nbins, nodata=lon.nodata), rep=rep)
+    t2 = device_raster(lon.dem, lon.rows, lon.cols)
+    assert (gpu_hist(t2, lon.gt, P2, lon.nbins, 128, lon.cols, nodata=lon.nodata, rep=rep) == H2).all()

@@ -253,3 +253,22 @@ def test_zonal_stats_from_histogram_match_cells():
         s2 = int((b * b).sum())
         assert st[k, 5] == np.int64(np.uint64(s2 & ((1 << 64) - 1)).view(np.int64)) and st[k, 6] == s2 >> 64
         assert st[k, 7] == np.unique(b).size
+
+
+def test_representative_point_offsets():
+    """SURVEY §8f-3 ('it is possible to use some other points (e.g., corners ...)').
+    With gt = (0,1,0,20,0,-1) and the point (c + 0, r + 1), cell (r, c) is represented by the
+    integer point (c, 19 - r).  Right triangle (0,0),(8,0),(0,8), half-open rule: the left leg
+    (x = 0) is never crossed from x >= 0, the hypotenuse is crossed iff x < 8 - y, y in [0, 8):
+    sum_{y=0..7} (8 - y) = 36 integer points (vs 28 cell centres).  Rectangle x in [2, 9],
+    y in [3, 7]: x in {2..8} (7) x y in {3..6} (4) = 28 with corners too."""
+    R = np.zeros((20, 24), np.int16)
+    gt = (0.0, 1.0, 0.0, 20.0, 0.0, -1.0)
+    P = from_rings([[(np.array([0.0, 8, 0]), np.array([0.0, 0, 8]))],
+                    [(np.array([2.0, 9, 9, 2]), np.array([3.0, 3, 7, 7]))]])
+    bins = oracle.make_bins(1)
+    for fn in (oracle.o0, oracle.o1):
+        assert [int(v) for v in fn(R, gt, P, bins, rep=(0.0, 1.0))[:, 0]] == [36, 28]
+        assert [int(v) for v in fn(R, gt, P, bins)[:, 0]] == [28, 28]
+    # centre == explicit (0.5, 0.5)
+    assert (oracle.o1(R, gt, P, bins, rep=(0.5, 0.5)) == oracle.o1(R, gt, P, bins)).all()
