@@ -205,6 +205,8 @@ def main():
     ap.add_argument("--path", default="fused", choices=["fused", "four_step"],
                     help="fused: step 2 + zh_fused_update (steps 1+3+4 fused, SURVEY §8f-1); four_step: 2,1,3,4")
     ap.add_argument("--no-other", action="store_true", help="skip timing the other path")
+    ap.add_argument("--equal-shards", action="store_true",
+                    help="N > 1: equal tile-row strips instead of the work-balanced plan (zh_plan_rows)")
     args = ap.parse_args()
 
     from synth.configs import CONFIGS
@@ -220,7 +222,7 @@ def main():
     import torch.distributed as dist
 
     from paper_conf_ipps_zhangw14_b200 import zh
-    from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms, shard_rows
+    from paper_conf_ipps_zhangw14_b200.dist import plan_shards, reduce_histograms
     from synth.dem import fill_device
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -246,7 +248,8 @@ def main():
     P = cfg.polygons()
     log(f"polygons: {P.n_poly} polys {P.n_vert} vertices ({time.perf_counter() - t_setup:.1f}s)")
     T = cfg.tile
-    r0, r1 = shard_rows(cfg.rows, T, world, rank)
+    bounds = plan_shards(cfg.rows, cfg.cols, cfg.gt, P, T, world, balanced=not args.equal_shards)
+    r0, r1 = bounds[rank], bounds[rank + 1]
     nrows = r1 - r0
     pitch = (cfg.cols + 7) // 8 * 8
     stream = torch.cuda.current_stream()
@@ -397,7 +400,8 @@ def main():
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
                 "data": "synthetic (fractal int16 DEM + jagged Voronoi counties, seeded)",
                 "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert,
-                               parallelism=f"tile-row shards x{world}" + (" (shared GPU, gloo)" if shared else ""),
+                               parallelism=f"tile-row shards x{world}" + (" (shared GPU, gloo)" if shared else "")
+                               + ("" if world == 1 else (" equal" if args.equal_shards else " work-balanced")),
                                l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA"),
                 "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
                 "clocks": clocks, "path": path, "steps_detail": steps_detail, "other_path": other,

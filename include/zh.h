@@ -184,6 +184,16 @@ zh_status zh_run(zh_ctx ctx, void* host_out);
 #define ZH_NSTATS 8
 zh_status zh_zonal_stats(zh_ctx ctx, int64_t* host_stats, int64_t** dptr);
 
+/* Work-balanced multi-GPU decomposition (the paper's future work on load
+ * balancing across nodes, §IV.C): split the raster's rows into n_shards contiguous
+ * ranges of WHOLE tile rows with about equal estimated work, from step 2's pair lists over the
+ * full raster (geometry only: raster values are not read; raster->data, row0, nrows and on_host
+ * are ignored).  row_bounds receives n_shards + 1 row indices (0 = first, rows = last); shard s
+ * holds rows [row_bounds[s], row_bounds[s+1]) (possibly empty).  shard_cost (may be NULL)
+ * receives the estimated cost of each shard (arbitrary units).  Runs on options->stream; syncs. */
+zh_status zh_plan_rows(const zh_raster* raster, const zh_polygons* polys, const zh_options* options,
+                       int32_t n_shards, int64_t* row_bounds, double* shard_cost);
+
 /* BORROWED device pointer to the output ([n_poly][nbins], uint64 or uint32) — e.g. for an
  * NCCL reduce across shards.  *n = n_poly * nbins elements. */
 zh_status zh_output_device(zh_ctx ctx, void** dptr, int64_t* n);

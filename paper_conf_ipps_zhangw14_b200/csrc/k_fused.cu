@@ -148,6 +148,35 @@ __global__ void __launch_bounds__(512, 3) k_fused_pure(PureP f) {
   pure_tile_body<kMode, kU64>(f, blockIdx.x, sh);
 }
 
+// ---- work-balanced shard planning: estimated cost of every tile row of the
+// raster from step 2's pair lists — cells of inside pairs (read once, histogrammed) and cells of
+// intersecting pairs (read per pair, tested) plus a fixed cost per intersecting pair.  Weights
+// are the measured per-cell times of the fused kernels.
+__global__ void k_row_cost(const int2* __restrict__ inside, int64_t n_inside, const int2* __restrict__ isect,
+                           int64_t n_isect, RasterP rp, double w_in, double w_x, double w_pair,
+                           double* __restrict__ row_cost) {
+  const int64_t n = n_inside + n_isect;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const bool in = i < n_inside;
+    const int tile = in ? inside[i].x : isect[i - n_inside].x;
+    const double cells = (double)tile_cells(rp, tile);
+    atomicAdd(&row_cost[tile / rp.TC], in ? w_in * cells : w_x * cells + w_pair);
+  }
+}
+
+cudaError_t launch_row_cost(Ctx& c, double* d_row_cost) {
+  cudaMemsetAsync(d_row_cost, 0, sizeof(double) * (size_t)c.rp.TRn, c.stream);
+  const int64_t n = c.n_inside + c.n_isect;
+  if (n > 0) {
+    int64_t b = (n + 255) / 256;
+    if (b > 148 * 32) b = 148 * 32;
+    k_row_cost<<<(unsigned)b, 256, 0, c.stream>>>(c.d_inside.as<int2>(), c.n_inside, c.d_isect.as<int2>(),
+                                                   c.n_isect, c.rp, 0.37, 0.53, 2000.0 * 0.37, d_row_cost);
+    c.launches += 1;
+  }
+  return cudaGetLastError();
+}
+
 static int grid_for(int64_t n, int threads) {
   int64_t b = (n + threads - 1) / threads;
   if (b > 148 * 32) b = 148 * 32;

@@ -366,6 +366,69 @@ extern "C" zh_status zh_zonal_stats(zh_ctx h, int64_t* host_stats, int64_t** dpt
   return ZH_OK;
 }
 
+extern "C" zh_status zh_plan_rows(const zh_raster* r, const zh_polygons* p, const zh_options* o, int32_t n_shards,
+                                  int64_t* row_bounds, double* shard_cost) {
+  if (!r || !p || !o || !row_bounds) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  if (n_shards < 1) return fail(ZH_ERR_INVALID_ARG, "n_shards must be >= 1");
+  // Geometry only: the raster values are never read by step 2, so a placeholder pointer stands in
+  // for the data and a single bin for the histograms.
+  zh_raster g = *r;
+  g.row0 = 0;
+  g.nrows = r->rows;
+  g.on_host = 0;
+  g.pitch = (r->cols + 7) / 8 * 8;
+  g.data = reinterpret_cast<const int16_t*>(static_cast<uintptr_t>(256));
+  zh_bins b1 = {0, 1, 1, 0, 0, 0};
+  zh_options go = *o;
+  go.out_u64 = 1;
+  go.force_isect = 0;
+  go.fused = 0;
+  zh_ctx h = nullptr;
+  zh_status s = zh_create(&h, &g, p, &b1, &go);
+  if (s != ZH_OK) return s;
+  Ctx* c = C(h);
+  const int64_t TR = c->rp.TRn;
+  std::vector<double> cost(TR > 0 ? TR : 1, 0.0);
+  s = zh_pair_tiles(h, nullptr, nullptr);
+  if (s == ZH_OK) {
+    zh::DBuf d;
+    cudaError_t e = d.ensure(sizeof(double) * (size_t)(TR > 0 ? TR : 1));
+    if (e == cudaSuccess) e = zh::launch_row_cost(*c, d.as<double>());
+    if (e == cudaSuccess && TR > 0)
+      e = cudaMemcpyAsync(cost.data(), d.p, sizeof(double) * (size_t)TR, cudaMemcpyDeviceToHost, c->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+    d.release();
+    if (e != cudaSuccess) s = cuda_fail(e, "zh_plan_rows");
+  }
+  zh_destroy(h);
+  if (s != ZH_OK) return s;
+  // contiguous split of the tile rows at equal prefix cost; a small per-row floor keeps empty rows
+  // (ocean) from collapsing all of them into one shard
+  const int64_t T = o->tile;
+  double total = 0.0;
+  for (int64_t i = 0; i < TR; ++i) total += cost[i];
+  const double floor_cost = total > 0 ? 1e-3 * total / (double)TR : 1.0;
+  for (int64_t i = 0; i < TR; ++i) cost[i] += floor_cost;
+  total += floor_cost * (double)TR;
+  row_bounds[0] = 0;
+  double run = 0.0;
+  int64_t tr = 0;
+  for (int i = 1; i < n_shards; ++i) {
+    const double target = total * (double)i / (double)n_shards;
+    while (tr < TR && run + cost[tr] * 0.5 < target) run += cost[tr++];
+    row_bounds[i] = std::min(tr * T, r->rows);
+  }
+  row_bounds[n_shards] = r->rows;
+  if (shard_cost) {
+    for (int i = 0; i < n_shards; ++i) {
+      double sc = 0.0;
+      for (int64_t t = row_bounds[i] / T; t < (row_bounds[i + 1] + T - 1) / T && t < TR; ++t) sc += cost[t];
+      shard_cost[i] = sc;
+    }
+  }
+  return ZH_OK;
+}
+
 extern "C" zh_status zh_output_device(zh_ctx h, void** dptr, int64_t* n) {
   if (!h || !dptr) return fail(ZH_ERR_INVALID_ARG, "null argument");
   Ctx* c = C(h);

@@ -83,6 +83,7 @@ cudaError_t launch_pip(Ctx& c);
 cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
 cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
 cudaError_t launch_zonal_stats(Ctx& c, int64_t* dstats);  // k_stats.cu
+cudaError_t launch_row_cost(Ctx& c, double* d_row_cost);  // k_fused.cu (shard planning)
 
 size_t device_bytes(const Ctx& c);
 

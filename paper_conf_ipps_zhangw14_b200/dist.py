@@ -23,6 +23,18 @@ def shard_rows(rows: int, tile: int, world: int, rank: int) -> tuple[int, int]:
     return r0, r1
 
 
+def plan_shards(rows: int, cols: int, gt, polygons, tile: int, world: int, balanced: bool = True):
+    """Row bounds (world + 1) of the decomposition: equal whole-tile-row strips, or — balanced —
+    strips of about equal estimated work from step 2's pairs over the whole raster (zh_plan_rows,
+    SURVEY.md §8f-2; §IV.C notes that equal partitions leave nodes near the coast
+    with little step-4 work).  Every rank computes the same plan (deterministic)."""
+    if not balanced or world == 1:
+        return [shard_rows(rows, tile, world, r)[0] for r in range(world)] + [rows]
+    from . import zh
+    bounds, _ = zh.plan_rows(rows, cols, gt, polygons, world, tile=tile)
+    return [int(b) for b in bounds]
+
+
 def reduce_histograms(out, group=None, to_rank0: bool = False):
     """Sum the per-rank partial histograms in place.  `out` is the int64 (uint64 bits) or int32
     view of libzh's output; two's-complement sums are bit-identical to unsigned ones."""

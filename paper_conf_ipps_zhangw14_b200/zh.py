@@ -61,7 +61,7 @@ class zh_stats(ctypes.Structure):
 
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",
-           "zh_fused_update", "zh_zonal_stats",
+           "zh_fused_update", "zh_zonal_stats", "zh_plan_rows",
            "zh_run", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
            "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy"]
 
@@ -83,6 +83,8 @@ def _load():
         "zh_pip_update": (st, [vp]),
         "zh_fused_update": (st, [vp]),
         "zh_zonal_stats": (st, [vp, vp, vp]),
+        "zh_plan_rows": (st, [ctypes.POINTER(zh_raster), ctypes.POINTER(zh_polygons), ctypes.POINTER(zh_options), i32,
+                              vp, vp]),
         "zh_run": (st, [vp, vp]),
         "zh_output_device": (st, [vp, ctypes.POINTER(vp), ctypes.POINTER(i64)]),
         "zh_set_output": (st, [vp, vp]),
@@ -123,6 +125,29 @@ def _stream_handle(stream) -> int:
     if hasattr(stream, "cuda_stream"):
         return stream.cuda_stream
     return int(stream)
+
+
+def plan_rows(rows: int, cols: int, gt, polygons, n_shards: int, tile: int = 256, stream=None, rep=None):
+    """zh_plan_rows: row bounds (n_shards + 1) of a work-balanced tile-row decomposition and the
+    estimated cost per shard."""
+    r = zh_raster()
+    r.data = None
+    r.rows, r.cols, r.pitch, r.row0, r.nrows = rows, cols, (cols + 7) // 8 * 8, 0, rows
+    r.gt = (ctypes.c_double * 6)(*[float(g) for g in gt])
+    r.on_host = 0
+    pro = np.ascontiguousarray(polygons.poly_ring_off, dtype=np.int64)
+    rvo = np.ascontiguousarray(polygons.ring_vert_off, dtype=np.int64)
+    x = np.ascontiguousarray(polygons.x, dtype=np.float64)
+    y = np.ascontiguousarray(polygons.y, dtype=np.float64)
+    p = zh_polygons(pro.shape[0] - 1, rvo.shape[0] - 1, x.shape[0], pro.ctypes.data, rvo.ctypes.data,
+                    x.ctypes.data, y.ctypes.data)
+    o = zh_options(tile, 1, 0, 0, _stream_handle(stream), 0 if rep is None else 1, 0,
+                   0.5 if rep is None else float(rep[0]), 0.5 if rep is None else float(rep[1]))
+    bounds = np.zeros(n_shards + 1, dtype=np.int64)
+    cost = np.zeros(n_shards, dtype=np.float64)
+    _check(LIB.zh_plan_rows(ctypes.byref(r), ctypes.byref(p), ctypes.byref(o), n_shards, bounds.ctypes.data,
+                            cost.ctypes.data))
+    return bounds, cost
 
 
 class _CAI:

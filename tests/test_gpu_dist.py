@@ -89,3 +89,39 @@ def test_two_ranks_reduce_to_oracle(cuda_device, cfg_name):
         assert (four == fused).all()
         for k in rows:
             assert (fused[k] == want[k]).all(), (rank, k)
+
+
+def test_plan_rows_balanced_shards(cuda_device):
+    """zh_plan_rows gives contiguous whole-tile-row shards; the shards of the tiny
+    config sum to the single-shard result; on CONUS the estimated costs are balanced."""
+    import torch
+
+    from paper_conf_ipps_zhangw14_b200 import zh
+    from paper_conf_ipps_zhangw14_b200.dist import plan_shards
+    from synth.configs import CONUS, TINY
+    from synth.dem import fill_device
+    cfg = TINY
+    P = cfg.polygons()
+    pitch = cfg.cols
+    full = torch.empty((cfg.rows, pitch), dtype=torch.int16, device="cuda")
+    fill_device(cfg.dem, cfg.cols, full.data_ptr(), 0, 0, cfg.rows, cfg.cols, pitch,
+                torch.cuda.current_stream().cuda_stream)
+    with zh.ZonalHistogram(full, cfg.gt, P, cfg.nbins, tile=64, nodata=cfg.nodata) as z:
+        want = z.run()
+    for n in (2, 3, 5):
+        b = plan_shards(cfg.rows, cfg.cols, cfg.gt, P, 64, n)
+        assert b[0] == 0 and b[-1] == cfg.rows and all(x <= y for x, y in zip(b, b[1:]))
+        assert all(x % 64 == 0 for x in b[:-1])
+        acc = np.zeros_like(want)
+        for s in range(n):
+            if b[s + 1] == b[s]:
+                continue
+            with zh.ZonalHistogram(full[b[s]:b[s + 1]], cfg.gt, P, cfg.nbins, tile=64, rows=cfg.rows, row0=b[s],
+                                   nodata=cfg.nodata) as z:
+                acc += z.run()
+        assert (acc == want).all()
+    C = CONUS
+    PC = C.polygons()
+    bounds, cost = zh.plan_rows(C.rows, C.cols, C.gt, PC, 8, tile=C.tile)
+    assert bounds[0] == 0 and bounds[-1] == C.rows
+    assert cost.max() / cost.mean() < 1.15, cost
