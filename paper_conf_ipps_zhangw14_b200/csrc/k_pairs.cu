@@ -58,14 +58,19 @@ __device__ __forceinline__ int2 straddle_rows(const Geo& g, double ya, double yb
 }
 
 // One CTA per polygon: for every vertex v of its rings, the edge v -> next(v) (implicit closure) in
-// canonical orientation, its exact straddled row interval within the shard, its polygon and the
-// number of tile rows it spans.  (Rings are contiguous, so no search is needed.)
+// canonical orientation and its exact straddled row interval within the shard; the number of
+// (edge, tile row) band entries is added to *n_entries.  Polygons whose tile rectangle misses the
+// shard (empty MBB) are skipped: nothing downstream reads their edges.  (Rings are contiguous, so
+// no search is needed.)
 __global__ void __launch_bounds__(256) k_edges(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
                                                const double* __restrict__ x, const double* __restrict__ y, Geo g,
-                                               int64_t rA, int64_t rB, int T, Edge* __restrict__ edges,
-                                               int2* __restrict__ erows, int32_t* __restrict__ epoly,
-                                               int32_t* __restrict__ espan) {
+                                               int64_t rA, int64_t rB, int T, const int4* __restrict__ mbb,
+                                               Edge* __restrict__ edges, int2* __restrict__ erows,
+                                               int64_t* __restrict__ n_entries) {
   const int k = blockIdx.x;
+  const int4 m = mbb[k];
+  if (m.x > m.y) return;
+  int span = 0;
   for (int ring = pro[k]; ring < pro[k + 1]; ++ring) {
     const int a = rvo[ring], b = rvo[ring + 1];
     for (int v = a + threadIdx.x; v < b; v += blockDim.x) {
@@ -77,10 +82,12 @@ __global__ void __launch_bounds__(256) k_edges(const int32_t* __restrict__ pro, 
       edges[v] = e;
       const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
       erows[v] = rr;
-      epoly[v] = k;
-      espan[v] = (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
+      span += (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
     }
   }
+  for (int o = 16; o > 0; o >>= 1) span += __shfl_xor_sync(0xffffffffu, span, o);
+  if ((threadIdx.x & 31) == 0 && span) atomicAdd(reinterpret_cast<unsigned long long*>(n_entries),
+                                                 (unsigned long long)span);
 }
 
 // One CTA per polygon: MBB of its vertices -> covered tile rectangle (global tile indices),
@@ -186,13 +193,17 @@ __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ 
 // exact parity is constant on it, and every straddling edge is >= 1 cell left/right of its
 // centres, so the computed parity equals the exact one at every centre.
 // class: 0 = not yet classified, 1 = inside, 2 = intersect, 3 = outside.
-__global__ void k_mark(const Edge* __restrict__ edges, const int32_t* __restrict__ epoly, int V, Geo g,
-                       RasterP rp, const int4* __restrict__ mbb, const int64_t* __restrict__ cand_off,
-                       uint8_t* __restrict__ cls) {
-  for (int v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
-    const int k = epoly[v];
-    const int4 m = mbb[k];
-    if (m.x > m.y) continue;
+__global__ void __launch_bounds__(256) k_mark(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                              const Edge* __restrict__ edges, Geo g, RasterP rp,
+                                              const int4* __restrict__ mbb, const int64_t* __restrict__ cand_off,
+                                              uint8_t* __restrict__ cls) {
+  const int k = blockIdx.x;
+  const int4 m = mbb[k];
+  if (m.x > m.y) return;
+  const int wk = m.y - m.x + 1;
+  const int64_t base = cand_off[k];
+  const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
+  for (int v = vb + threadIdx.x; v < ve; v += blockDim.x) {
     const Edge e = edges[v];
     double ca = (fmin(e.xa, e.xb) - g.gt0) / g.gt1, cb = (fmax(e.xa, e.xb) - g.gt0) / g.gt1;
     if (ca > cb) { double t = ca; ca = cb; cb = t; }
@@ -205,8 +216,6 @@ __global__ void k_mark(const Edge* __restrict__ edges, const int32_t* __restrict
     if (clo > chi || rlo > rhi) continue;
     const int tc_lo = (int)((int64_t)clo / rp.T), tc_hi = (int)((int64_t)chi / rp.T);
     const int tr_lo = (int)((int64_t)rlo / rp.T), tr_hi = (int)((int64_t)rhi / rp.T);
-    const int wk = m.y - m.x + 1;
-    const int64_t base = cand_off[k];
     for (int tr = tr_lo; tr <= tr_hi; ++tr)
       for (int tc = tc_lo; tc <= tc_hi; ++tc) cls[base + (int64_t)(tr - m.z) * wk + (tc - m.x)] = 2;
   }
@@ -300,11 +309,9 @@ __global__ void k_compact(const uint8_t* __restrict__ cls, const uint64_t* __res
   }
 }
 
-__global__ void k_totals1(const int64_t* cand_off, const int64_t* band_base, const int32_t* espan_sum, int P,
-                          int64_t* out) {
+__global__ void k_totals1(const int64_t* cand_off, const int64_t* band_base, int P, int64_t* out) {
   out[0] = cand_off[P];
   out[1] = band_base[P];
-  out[2] = espan_sum[0];
 }
 
 static int grid_for(int64_t n, int threads) {
@@ -327,7 +334,6 @@ static cudaError_t excl_scan(Ctx& c, const T* in, T* out, int64_t n) {
 
 }  // namespace zh
 
-#include <cub/device/device_reduce.cuh>
 
 namespace zh {
 
@@ -336,8 +342,6 @@ cudaError_t launch_pairs_phase1(Ctx& c) {
   const int V = c.V, P = c.P;
   if ((e = c.d_edges.ensure(sizeof(Edge) * (size_t)V)) != cudaSuccess) return e;
   if ((e = c.d_erows.ensure(sizeof(int2) * (size_t)V)) != cudaSuccess) return e;
-  if ((e = c.d_epoly.ensure(sizeof(int32_t) * (size_t)V)) != cudaSuccess) return e;
-  if ((e = c.d_espan.ensure(sizeof(int32_t) * ((size_t)V + 1))) != cudaSuccess) return e;
   if ((e = c.d_mbb.ensure(sizeof(int4) * (size_t)P)) != cudaSuccess) return e;
   if ((e = c.d_ncand.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
   if ((e = c.d_nband.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
@@ -345,38 +349,25 @@ cudaError_t launch_pairs_phase1(Ctx& c) {
   if ((e = c.d_band_base.ensure(sizeof(int64_t) * ((size_t)P + 1))) != cudaSuccess) return e;
   if ((e = c.d_counts.ensure(sizeof(int64_t) * 8)) != cudaSuccess) return e;
   const int64_t rA = c.rp.row0, rB = c.rp.row0 + c.rp.nrows;
-  if (V > 0) {
-    k_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
-                                     c.d_y.as<double>(), c.geo, rA, rB, c.rp.T, c.d_edges.as<Edge>(),
-                                     c.d_erows.as<int2>(), c.d_epoly.as<int32_t>(), c.d_espan.as<int32_t>());
-    c.launches += 1;
-  }
   // one trailing zero so that the exclusive scans over P + 1 entries end with the totals
   cudaMemsetAsync(c.d_ncand.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
   cudaMemsetAsync(c.d_nband.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
+  cudaMemsetAsync(c.d_counts.p, 0, sizeof(int64_t) * 8, c.stream);
   if (P > 0) {
     k_mbb<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
                                    c.d_y.as<double>(), c.geo, c.rp, c.d_mbb.as<int4>(), c.d_ncand.as<int64_t>(),
                                    c.d_nband.as<int64_t>());
     c.launches += 1;
   }
+  if (V > 0) {
+    k_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
+                                     c.d_y.as<double>(), c.geo, rA, rB, c.rp.T, c.d_mbb.as<int4>(),
+                                     c.d_edges.as<Edge>(), c.d_erows.as<int2>(), c.d_counts.as<int64_t>() + 2);
+    c.launches += 1;
+  }
   if ((e = excl_scan<int64_t>(c, c.d_ncand.as<int64_t>(), c.d_cand_off.as<int64_t>(), P + 1)) != cudaSuccess) return e;
   if ((e = excl_scan<int64_t>(c, c.d_nband.as<int64_t>(), c.d_band_base.as<int64_t>(), P + 1)) != cudaSuccess) return e;
-  // espan total (int32 is enough: < 2^31 checked on the host afterwards via int64 sum below)
-  int32_t* sum_out = c.d_espan.as<int32_t>() + V;  // scratch slot
-  if (V > 0) {
-    size_t need = 0;
-    if ((e = cub::DeviceReduce::Sum(nullptr, need, c.d_espan.as<int32_t>(), sum_out, V, c.stream)) != cudaSuccess)
-      return e;
-    if ((e = c.d_cub.ensure(need)) != cudaSuccess) return e;
-    size_t have = c.d_cub.bytes;
-    c.launches += 2;  // CUB reduce kernels
-    if ((e = cub::DeviceReduce::Sum(c.d_cub.p, have, c.d_espan.as<int32_t>(), sum_out, V, c.stream)) != cudaSuccess)
-      return e;
-  } else {
-    cudaMemsetAsync(sum_out, 0, sizeof(int32_t), c.stream);
-  }
-  k_totals1<<<1, 1, 0, c.stream>>>(c.d_cand_off.as<int64_t>(), c.d_band_base.as<int64_t>(), sum_out, P,
+  k_totals1<<<1, 1, 0, c.stream>>>(c.d_cand_off.as<int64_t>(), c.d_band_base.as<int64_t>(), P,
                                    c.d_counts.as<int64_t>());
   c.launches += 1;
   return cudaGetLastError();
@@ -420,8 +411,8 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
     } else {
       cudaMemsetAsync(c.d_class.p, 0, (size_t)nc, c.stream);
       if (V > 0) {
-        k_mark<<<grid_for(V, 256), 256, 0, c.stream>>>(c.d_edges.as<Edge>(), c.d_epoly.as<int32_t>(), V, c.geo,
-                                                      c.rp, c.d_mbb.as<int4>(),
+        k_mark<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_edges.as<Edge>(), c.geo,
+                                       c.rp, c.d_mbb.as<int4>(),
                                                       c.d_cand_off.as<int64_t>(), c.d_class.as<uint8_t>());
         c.launches += 1;
       }

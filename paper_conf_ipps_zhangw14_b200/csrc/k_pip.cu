@@ -26,12 +26,12 @@
 
 namespace zh {
 
-template <int kMode, bool kU64>
+template <int kMode, bool kU64, bool kRep>
 __global__ void __launch_bounds__(256) k_pip(PipP p) {
   if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
   extern __shared__ __align__(16) uint32_t sh[];
   __shared__ LongQ lq;
-  pip_pair_body<kMode, kU64>(p, blockIdx.x, sh, &lq);
+  pip_pair_body<kMode, kU64, kRep>(p, blockIdx.x, sh, &lq);
 }
 
 cudaError_t launch_pip(Ctx& c) { return launch_pip_list(c, c.d_isect.as<int2>(), c.n_isect, nullptr); }
@@ -74,13 +74,17 @@ cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64
   const int threads = 256;
   void (*k)(PipP);
   const int mode = fast_bins_ok(c.bp) ? (p.fb.bias ? 4 : (c.bp.use_nodata ? 3 : 2)) : (c.bp.width == 1 ? 0 : 1);
+  const bool rep = !(c.geo.ox == 0.5 && c.geo.oy == 0.5);
+#define ZH_PIP_K(M) (c.out_u64 ? (rep ? k_pip<M, true, true> : k_pip<M, true, false>) \
+                               : (rep ? k_pip<M, false, true> : k_pip<M, false, false>))
   switch (mode) {
-    case 0: k = c.out_u64 ? k_pip<0, true> : k_pip<0, false>; break;
-    case 1: k = c.out_u64 ? k_pip<1, true> : k_pip<1, false>; break;
-    case 2: k = c.out_u64 ? k_pip<2, true> : k_pip<2, false>; break;
-    case 3: k = c.out_u64 ? k_pip<3, true> : k_pip<3, false>; break;
-    default: k = c.out_u64 ? k_pip<4, true> : k_pip<4, false>; break;
+    case 0: k = ZH_PIP_K(0); break;
+    case 1: k = ZH_PIP_K(1); break;
+    case 2: k = ZH_PIP_K(2); break;
+    case 3: k = ZH_PIP_K(3); break;
+    default: k = ZH_PIP_K(4); break;
   }
+#undef ZH_PIP_K
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k<<<(unsigned)grid, threads, smem, c.stream>>>(p);
   c.launches += 1;

@@ -200,7 +200,7 @@ extern "C" void zh_destroy(zh_ctx h) {
   Ctx* c = C(h);
   cudaStreamSynchronize(c->stream);
   zh::DBuf* bufs[] = {&c->raster_dev, &c->d_pro, &c->d_rvo, &c->d_x, &c->d_y, &c->d_edges, &c->d_erows,
-                      &c->d_epoly, &c->d_espan, &c->d_mbb, &c->d_ncand, &c->d_nband, &c->d_cand_off,
+                      &c->d_mbb, &c->d_ncand, &c->d_nband, &c->d_cand_off,
                       &c->d_band_base, &c->d_band_cnt, &c->d_band_off, &c->d_band_cur, &c->d_band_edges,
                       &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
@@ -215,7 +215,7 @@ extern "C" void zh_destroy(zh_ctx h) {
 
 size_t zh::device_bytes(const Ctx& c) {
   const zh::DBuf* bufs[] = {&c.raster_dev, &c.d_pro, &c.d_rvo, &c.d_x, &c.d_y, &c.d_edges, &c.d_erows,
-                            &c.d_epoly, &c.d_espan, &c.d_mbb, &c.d_ncand, &c.d_nband, &c.d_cand_off,
+                            &c.d_mbb, &c.d_ncand, &c.d_nband, &c.d_cand_off,
                             &c.d_band_base, &c.d_band_cnt, &c.d_band_off, &c.d_band_cur, &c.d_band_edges,
                             &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,

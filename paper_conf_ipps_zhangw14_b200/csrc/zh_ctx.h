@@ -49,7 +49,7 @@ struct Ctx {
   int32_t P = 0, R = 0, V = 0;
   DBuf d_pro, d_rvo, d_x, d_y;
   // step 2 products
-  DBuf d_edges, d_erows, d_epoly, d_espan, d_mbb, d_ncand, d_nband, d_cand_off, d_band_base;
+  DBuf d_edges, d_erows, d_mbb, d_ncand, d_nband, d_cand_off, d_band_base;
   DBuf d_band_cnt, d_band_off, d_band_cur, d_band_edges, d_class, d_flags, d_flag_pos;
   DBuf d_inside, d_isect, d_counts, d_cub;
   // fused path lists (k_fused.cu)

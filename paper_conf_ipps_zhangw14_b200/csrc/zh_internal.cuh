@@ -21,11 +21,16 @@ struct Geo {
   double ox, oy;
 };
 
+// kRep = false: the centre (0.5 as an immediate — the hot kernels are instantiated for it, the
+// runtime offsets cost ~12 % in k_pip); kRep = true: the runtime offsets g.ox, g.oy.  Both give
+// identical values when the offsets are 0.5.
+template <bool kRep = true>
 __device__ __forceinline__ double col_centre(const Geo& g, int64_t c) {
-  return __dadd_rn(g.gt0, __dmul_rn(__dadd_rn((double)c, g.ox), g.gt1));
+  return __dadd_rn(g.gt0, __dmul_rn(__dadd_rn((double)c, kRep ? g.ox : 0.5), g.gt1));
 }
+template <bool kRep = true>
 __device__ __forceinline__ double row_centre(const Geo& g, int64_t r) {
-  return __dadd_rn(g.gt3, __dmul_rn(__dadd_rn((double)r, g.oy), g.gt5));
+  return __dadd_rn(g.gt3, __dmul_rn(__dadd_rn((double)r, kRep ? g.oy : 0.5), g.gt5));
 }
 
 // Canonical edge (ya <= yb), Fig. 5 predicate in lower-endpoint-first orientation (R8).

@@ -24,6 +24,7 @@ struct TileGeom {
   bool s;          // gt1 > 0: xc increases with the column
 };
 
+template <bool kRep = true>
 __device__ __forceinline__ TileGeom tile_geom(const RasterP& rp, const Geo& g, int tile) {
   TileGeom t;
   const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
@@ -31,7 +32,7 @@ __device__ __forceinline__ TileGeom tile_geom(const RasterP& rp, const Geo& g, i
   t.h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - t.r0);
   t.c0 = (int64_t)tc * rp.T;
   t.w = (int)min((int64_t)rp.T, rp.cols - t.c0);
-  const double xa = col_centre(g, t.c0), xb = col_centre(g, t.c0 + t.w - 1);
+  const double xa = col_centre<kRep>(g, t.c0), xb = col_centre<kRep>(g, t.c0 + t.w - 1);
   t.xlo_t = fmin(xa, xb);
   t.xhi_t = fmax(xa, xb);
   t.half = 0.5 * fabs(g.gt1);
@@ -40,17 +41,19 @@ __device__ __forceinline__ TileGeom tile_geom(const RasterP& rp, const Geo& g, i
 }
 
 // One (edge, row) crossing: flip the bits of D that record {c : xc(c) < xi}.
+template <bool kRep>
 __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr, const Edge& e, int64_t r,
                                              int64_t rlo, const Geo& g, const TileGeom& t) {
   const int w = t.w;
-  const double yc = row_centre(g, r);
+  const double yc = row_centre<kRep>(g, r);
   const double xi = intercept(e, yc);
   const double est = (xi - g.gt0) / g.gt1 - g.ox - (double)t.c0;
   int64_t ei;
   if (!(est > 0.0)) ei = 0;
   else if (est > (double)w) ei = w;
   else ei = (int64_t)ceil(est);
-  const int64_t jb = first_false(0, w, ei, [&](int64_t j) { return (col_centre(g, t.c0 + j) < xi) == t.s; });
+  const int64_t jb =
+      first_false(0, w, ei, [&](int64_t j) { return (col_centre<kRep>(g, t.c0 + j) < xi) == t.s; });
   const int lr = (int)(r - rlo);
   if (jb > 0) atomicXor(&bm[lr * wpr + (int)(jb >> 5)], 1u << (jb & 31));
   if (!t.s) atomicXor(&bm[lr * wpr + (w >> 5)], 1u << (w & 31));
@@ -69,6 +72,7 @@ struct LongQ {
 // Step 1 of the header comment for band edges [e0, e1) into bm (rows [rlo, rhi), wpr words per
 // row, zeroed by the caller).  Block-strided over the band's edges; `q` must hold q->n = 0, made
 // visible by a barrier, before the first call; the function leaves it so and ends with a barrier.
+template <bool kRep>
 __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, int wpr, int e0, int e1,
                                                     const int32_t* __restrict__ band_edges,
                                                     const Edge* __restrict__ edges, const int2* __restrict__ erows,
@@ -94,7 +98,7 @@ __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, i
     if (all) {
       for (int64_t r = ra; r < rb; ++r) atomicXor(&bm[(int)(r - rlo) * wpr + (w >> 5)], 1u << (w & 31));
     } else {
-      for (int64_t r = ra; r < rb; ++r) crossing_row(bm, wpr, e, r, rlo, g, t);
+      for (int64_t r = ra; r < rb; ++r) crossing_row<kRep>(bm, wpr, e, r, rlo, g, t);
     }
   }
   __syncthreads();
@@ -108,7 +112,7 @@ __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, i
       for (int r = it.y + lane; r < it.z; r += 32) atomicXor(&bm[(int)(r - rlo) * wpr + (w >> 5)], 1u << (w & 31));
     } else {
       const Edge e = edges[it.x];
-      for (int r = it.y + lane; r < it.z; r += 32) crossing_row(bm, wpr, e, r, rlo, g, t);
+      for (int r = it.y + lane; r < it.z; r += 32) crossing_row<kRep>(bm, wpr, e, r, rlo, g, t);
     }
   }
   __syncthreads();

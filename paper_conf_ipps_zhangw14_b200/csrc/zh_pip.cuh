@@ -31,7 +31,7 @@ size_t pip_smem(const Ctx& c, const PipP& p);
 // `sh` holds hist_words(nbins) + rc * wpr words; `lq` must hold n = 0 (published by a barrier before
 // the first crossing phase — the body's first barrier does that).
 // kMode as in k_tile_hist: 0/1 generic (w1 / w>1), 2 + kForm packed.
-template <int kMode, bool kU64>
+template <int kMode, bool kU64, bool kRep>
 __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, uint32_t* __restrict__ sh,
                                               LongQ* lqp) {
   LongQ& lq = *lqp;
@@ -44,7 +44,7 @@ __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, u
 
   const int2 pr = p.isect[pair_idx];
   const int tile = pr.x, k = pr.y;
-  const TileGeom t = tile_geom(rp, g, tile);
+  const TileGeom t = tile_geom<kRep>(rp, g, tile);
   const int64_t r0 = t.r0, c0 = t.c0;
   const int h = t.h, w = t.w;
   const int4 m = p.mbb[k];
@@ -66,7 +66,7 @@ __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, u
     const int64_t rlo = r0 + cr, rhi = rlo + ch;  // global rows of this chunk
     for (int i = threadIdx.x; i < ch * p.wpr; i += blockDim.x) bm[i] = 0;
     __syncthreads();
-    crossings_to_bitmap(bm, p.wpr, e0, e1, p.band_edges, p.edges, p.erows, g, t, rlo, rhi, &lq);
+    crossings_to_bitmap<kRep>(bm, p.wpr, e0, e1, p.band_edges, p.edges, p.erows, g, t, rlo, rhi, &lq);
     suffix_xor_rows(bm, p.wpr, ch);
     __syncthreads();
     // ---- cells: stream the chunk's rows, count inside cells (fully-outside vectors are not read)
