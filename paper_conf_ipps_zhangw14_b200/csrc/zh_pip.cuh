@@ -122,11 +122,16 @@ __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, u
   // ---- flush the pair's histogram
   const int nbins = p.bp.nbins;
   const int64_t orow = (int64_t)k * nbins;
-  for (int b = threadIdx.x; b < nbins; b += blockDim.x) {
-    const uint32_t v = hist[kOff + b];
-    if (v) {
-      if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(p.out) + orow + b, (unsigned long long)v);
-      else atomicAdd(reinterpret_cast<uint32_t*>(p.out) + orow + b, v);
+  for (int b = threadIdx.x * 4; b < nbins; b += blockDim.x * 4) {  // 16-byte reads, zero vectors skipped
+    const uint4 v = *reinterpret_cast<const uint4*>(&hist[kOff + b]);
+    if (!(v.x | v.y | v.z | v.w)) continue;
+    const uint32_t vs[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (vs[q] && b + q < nbins) {
+        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(p.out) + orow + b + q, (unsigned long long)vs[q]);
+        else atomicAdd(reinterpret_cast<uint32_t*>(p.out) + orow + b + q, vs[q]);
+      }
     }
   }
 }
