@@ -1,0 +1,25 @@
+"""compute-sanitizer memcheck / racecheck / synccheck over small runs of every libzh kernel
+(tools/sanitize.py: both paths, aligned and ragged tiles, zonal statistics).  The printed
+pip_test_kernel of the paper races on the histogram; this build must not."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer(cuda_device, tool):
+    exe = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(exe):
+        pytest.skip("compute-sanitizer not available")
+    r = subprocess.run([exe, "--tool", tool, "--error-exitcode", "3", sys.executable,
+                        os.path.join(ROOT, "tools", "sanitize.py")], capture_output=True, text=True, timeout=900)
+    out = r.stdout + r.stderr
+    assert r.returncode == 0, out[-3000:]
+    assert "sanitize run ok" in out
+    assert ("0 errors" in out) or ("0 hazards" in out), out[-2000:]

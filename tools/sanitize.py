@@ -1,0 +1,23 @@
+"""Small end-to-end runs for compute-sanitizer (memcheck / racecheck / synccheck): tiny config,
+both paths, a ragged tile size, and the zonal statistics.  python tools/sanitize.py"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_ipps_zhangw14_b200 import zh  # noqa: E402
+from synth.configs import TINY as cfg  # noqa: E402
+from synth.dem import fill_device  # noqa: E402
+
+P = cfg.polygons()
+t = torch.empty((cfg.rows, cfg.cols), dtype=torch.int16, device="cuda")
+fill_device(cfg.dem, cfg.cols, t.data_ptr(), 0, 0, cfg.rows, cfg.cols, cfg.cols, torch.cuda.current_stream().cuda_stream)
+res = []
+for tile, fused in ((128, False), (128, True), (100, True), (100, False)):
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=tile, nodata=cfg.nodata, fused=fused) as z:
+        res.append(z.run())
+        z.zh_zonal_stats()
+assert all((r == res[0]).all() for r in res)
+print("sanitize run ok", int(res[0].sum()))
