@@ -300,3 +300,14 @@ def test_representative_points(tiny, cuda_device, rep):
     H2 = oracle.o1(R2, lon.gt, P2, oracle.make_bins(lon.nbins, nodata=lon.nodata), rep=rep)
     t2 = device_raster(lon.dem, lon.rows, lon.cols)
     assert (gpu_hist(t2, lon.gt, P2, lon.nbins, 128, lon.cols, nodata=lon.nodata, rep=rep) == H2).all()
+
+
+@pytest.mark.parametrize("nbins,lo,width", [(20000, -10000, 1), (49152, -32768, 1), (3000, -400, 2)])
+def test_large_and_generic_histograms(tiny, cuda_device, nbins, lo, width):
+    """Histograms beyond the packed 16x2 path (nbins > 16000, width > 1): the generic per-cell
+    path and the shared-memory budget logic (49,152 bins = 192 KB per CTA)."""
+    cfg, P, R, _ = tiny
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(nbins, lo=lo, width=width, nodata=cfg.nodata))
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    G = gpu_hist(t, cfg.gt, P, nbins, 128, cfg.cols, lo=lo, width=width, nodata=cfg.nodata)
+    assert (G == H).all()
