@@ -334,6 +334,9 @@ def main():
         steps_detail = {"step2_pair_tiles": {"ms": avg(lib_ms, "step2_pair_tiles")}}
     for name, (t, b) in kern.items():
         steps_detail[name] = {"ms": t, "alg_bytes": b, "alg_GBps": b / (t / 1000.0) / 1e9 if t else None}
+    if path == "fused":
+        # the parity bitmaps of the mixed pairs (FP64 crossing work), on a second stream beside k_fused_pure
+        steps_detail["k_parity(side stream)"] = {"ms": avg(lib_ms, "fused_parity_kernel")}
     dom = max(kern, key=lambda k: kern[k][0] or 0.0)
     dom_ms, dom_b = kern[dom]
     achieved = dom_b / (dom_ms / 1000.0) / 1e9

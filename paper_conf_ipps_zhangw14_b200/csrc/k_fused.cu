@@ -17,20 +17,29 @@
 #include "zh_pip.cuh"
 #include "zh_tilehist.cuh"
 
+#ifndef ZH_PAR_SIDE
+#define ZH_PAR_SIDE 0  // 1: k_parity on the side stream, beside k_fused_pure (measured slower: registers)
+#endif
+
 namespace zh {
 
-__global__ void k_mark_mixed(const int2* __restrict__ isect, int64_t n, uint8_t* __restrict__ mixed) {
+// pip_cnt[t] = #pairs of tile t for the cell-in-polygon kernel: its intersecting pairs, then (below)
+// the inside pairs of the tiles that have one (a tile is "mixed" iff it has an intersecting pair)
+__global__ void k_mark_mixed(const int2* __restrict__ isect, int64_t n, uint32_t* __restrict__ pip_cnt) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    mixed[isect[i].x] = 1;
+    atomicAdd(&pip_cnt[isect[i].x], 1u);
 }
 
 // inside pairs of pure tiles are counted per tile; inside pairs of mixed tiles are flagged "extra"
-__global__ void k_inside_split(const int2* __restrict__ inside, int64_t n, const uint8_t* __restrict__ mixed,
+// and join the tile's cell-in-polygon pairs (pip_cnt of a tile is either 0 throughout — pure — or
+// > 0 before and after this kernel's increments, so the test below does not race)
+__global__ void k_inside_split(const int2* __restrict__ inside, int64_t n, uint32_t* __restrict__ pip_cnt,
                                uint32_t* __restrict__ pure_cnt, uint32_t* __restrict__ extra) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const int t = inside[i].x;
-    if (mixed[t]) {
+    if (*(volatile uint32_t*)&pip_cnt[t]) {
       extra[i] = 1;
+      atomicAdd(&pip_cnt[t], 1u);
     } else {
       extra[i] = 0;
       atomicAdd(&pure_cnt[t], 1u);
@@ -79,26 +88,28 @@ __global__ void k_pure_tiles(const uint32_t* __restrict__ pure_cnt, int64_t n, c
                                                   (unsigned long long)cells);
 }
 
-// counts[1] = #pairs for the cell-in-polygon kernel, counts[3] = their tiles' cells
+// counts[1] = #pairs for the cell-in-polygon kernel, counts[3] = their tiles' cells.  The list is
+// grouped BY TILE (pip_off = exclusive scan of pip_cnt), so the 2-3 pairs that read the same mixed
+// tile run back to back and all but the first find its cells in L2 (grouped by polygon, as step 2
+// emits them, the L2 hit rate of k_pip was 15 %).
 __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, const int2* __restrict__ inside,
-                           int64_t n_inside, const uint32_t* __restrict__ extra, const uint32_t* __restrict__ extra_pos,
-                           RasterP rp, int2* __restrict__ pip, int64_t* __restrict__ counts) {
+                           int64_t n_inside, const uint32_t* __restrict__ extra, const uint32_t* __restrict__ pip_off,
+                           uint32_t* __restrict__ cursor, int64_t n_tiles, RasterP rp, int2* __restrict__ pip,
+                           int64_t* __restrict__ counts) {
   const int64_t n = n_isect + n_inside;
   int64_t cells = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int2 pr;
     if (i < n_isect) {
-      pip[i] = isect[i];
-      cells += tile_cells(rp, isect[i].x);
+      pr = isect[i];
     } else {
-      const int64_t j = i - n_isect;
-      if (extra[j]) {
-        pip[n_isect + extra_pos[j]] = inside[j];
-        cells += tile_cells(rp, inside[j].x);
-      }
-      if (j == n_inside - 1) counts[1] = n_isect + (int64_t)extra_pos[j] + extra[j];
+      if (!extra[i - n_isect]) continue;
+      pr = inside[i - n_isect];
     }
+    pip[pip_off[pr.x] + atomicAdd(&cursor[pr.x], 1u)] = pr;
+    cells += tile_cells(rp, pr.x);
   }
-  if (n_inside == 0 && blockIdx.x == 0 && threadIdx.x == 0) counts[1] = n_isect;
+  if (blockIdx.x == 0 && threadIdx.x == 0) counts[1] = (int64_t)pip_off[n_tiles];
   for (int o = 16; o > 0; o >>= 1) cells += __shfl_xor_sync(0xffffffffu, cells, o);
   if ((threadIdx.x & 31) == 0 && cells) atomicAdd(reinterpret_cast<unsigned long long*>(&counts[3]),
                                                   (unsigned long long)cells);
@@ -226,7 +237,8 @@ static void launch_pure(Ctx& c, size_t smem, unsigned grid) {
 cudaError_t launch_fused(Ctx& c) {
   cudaError_t e;
   const int64_t NT = c.n_tiles, NI = c.n_inside, NX = c.n_isect;
-  if ((e = c.d_mixed.ensure((size_t)NT + 16)) != cudaSuccess) return e;
+  if ((e = c.d_mixed.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_pip_cur.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pure_cnt.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pure_cur.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pure_pk.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
@@ -234,25 +246,26 @@ cudaError_t launch_fused(Ctx& c) {
   if ((e = c.d_pure_poly.ensure(sizeof(int32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
   if ((e = c.d_pure_tiles.ensure(sizeof(int32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
   if ((e = c.d_extra.ensure(sizeof(uint32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
-  if ((e = c.d_extra_pos.ensure(sizeof(uint32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
+  if ((e = c.d_extra_pos.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pip.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
   if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 4)) != cudaSuccess) return e;
   cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 4, c.stream);
   if (NT == 0 || NI + NX == 0) {
     if (c.timing)
-      for (int i = 10; i < 13; ++i) cudaEventRecord(c.ev[i], c.stream);
+      for (int i = 10; i < 16; ++i) cudaEventRecord(c.ev[i], c.stream);
     return cudaGetLastError();
   }
 
-  cudaMemsetAsync(c.d_mixed.p, 0, (size_t)NT, c.stream);
+  cudaMemsetAsync(c.d_mixed.p, 0, sizeof(uint32_t) * ((size_t)NT + 1), c.stream);
+  cudaMemsetAsync(c.d_pip_cur.p, 0, sizeof(uint32_t) * ((size_t)NT + 1), c.stream);
   cudaMemsetAsync(c.d_pure_cnt.p, 0, sizeof(uint32_t) * ((size_t)NT + 1), c.stream);
   cudaMemsetAsync(c.d_pure_cur.p, 0, sizeof(uint32_t) * ((size_t)NT + 1), c.stream);
   if (NX > 0) {
-    k_mark_mixed<<<grid_for(NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_mixed.as<uint8_t>());
+    k_mark_mixed<<<grid_for(NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_mixed.as<uint32_t>());
     c.launches += 1;
   }
   if (NI > 0) {
-    k_inside_split<<<grid_for(NI, 256), 256, 0, c.stream>>>(c.d_inside.as<int2>(), NI, c.d_mixed.as<uint8_t>(),
+    k_inside_split<<<grid_for(NI, 256), 256, 0, c.stream>>>(c.d_inside.as<int2>(), NI, c.d_mixed.as<uint32_t>(),
                                                            c.d_pure_cnt.as<uint32_t>(), c.d_extra.as<uint32_t>());
     c.launches += 1;
   }
@@ -270,18 +283,31 @@ cudaError_t launch_fused(Ctx& c) {
   k_pure_tiles<<<grid_for(NT, 256), 256, 0, c.stream>>>(c.d_pure_cnt.as<uint32_t>(), NT, c.d_pure_off.as<uint64_t>(),
                                                         c.rp, c.d_pure_tiles.as<int32_t>(), c.d_fcounts.as<int64_t>());
   c.launches += 1;
-  if (NI > 0) {
-    if ((e = excl_scan<uint32_t>(c, c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(), NI)) != cudaSuccess)
-      return e;
-  }
+  if ((e = excl_scan<uint32_t>(c, c.d_mixed.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(), NT + 1)) != cudaSuccess)
+    return e;
   k_pip_list<<<grid_for(NI + NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_inside.as<int2>(), NI,
                                                           c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(),
-                                                          c.rp, c.d_pip.as<int2>(), c.d_fcounts.as<int64_t>());
+                                                          c.d_pip_cur.as<uint32_t>(), NT, c.rp, c.d_pip.as<int2>(),
+                                                          c.d_fcounts.as<int64_t>());
   c.launches += 1;
 
   const int mode = fast_bins_ok(c.bp) ? (make_fast_bins(c.bp).bias ? 4 : (c.bp.use_nodata ? 3 : 2))
                                       : (c.bp.width == 1 ? 0 : 1);
-  // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
+  // mixed tiles, split form: the parity bitmaps of every cell-in-polygon pair are built on the side
+  // stream WHILE the pure-tile kernel streams the pure tiles (FP64-latency work beside HBM-bound
+  // work), then the cell kernel runs once both are done
+  const bool split = c.pip_split != 0;
+  if (split) {
+    if ((e = pip_prepare(c, NI + NX)) != cudaSuccess) return e;
+    cudaEventRecord(c.ev_fork, c.stream);
+    cudaStreamWaitEvent(c.side, c.ev_fork, 0);
+    if (c.timing) cudaEventRecord(c.ev[13], ZH_PAR_SIDE ? c.side : c.stream);
+    if ((e = launch_parity(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1,
+                           ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess)
+      return e;
+    if (c.timing) cudaEventRecord(c.ev[14], ZH_PAR_SIDE ? c.side : c.stream);
+    cudaEventRecord(c.ev_join, c.side);
+  }
   // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
   if (c.timing) cudaEventRecord(c.ev[10], c.stream);
   if (NI > 0) {
@@ -308,8 +334,18 @@ cudaError_t launch_fused(Ctx& c) {
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
   if (c.timing) cudaEventRecord(c.ev[11], c.stream);
-  // mixed tiles: every pair through the cell-in-polygon kernel
-  e = launch_pip_list(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1);
+  if (split) {
+    cudaStreamWaitEvent(c.stream, c.ev_join, 0);
+    if (c.timing) cudaEventRecord(c.ev[15], c.stream);
+    e = launch_pip_cells(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1);
+  } else {
+    if (c.timing) {
+      cudaEventRecord(c.ev[13], c.stream);
+      cudaEventRecord(c.ev[14], c.stream);
+      cudaEventRecord(c.ev[15], c.stream);
+    }
+    e = launch_pip_list(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1);
+  }
   if (c.timing) cudaEventRecord(c.ev[12], c.stream);
   return e;
 }

@@ -26,15 +26,46 @@
 
 namespace zh {
 
+#ifndef ZH_PIP_MINB
+#define ZH_PIP_MINB 6
+#endif
+#ifndef ZH_PIP_THREADS
+#define ZH_PIP_THREADS 256
+#endif
+constexpr int kPipThreads = ZH_PIP_THREADS;  // k_pip_cells
+
 template <int kMode, bool kU64, bool kRep>
-__global__ void __launch_bounds__(256) k_pip(PipP p) {
+__global__ void __launch_bounds__(256, ZH_PIP_MINB) k_pip(PipP p) {
   if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
   extern __shared__ __align__(16) uint32_t sh[];
   __shared__ LongQ lq;
   pip_pair_body<kMode, kU64, kRep>(p, blockIdx.x, sh, &lq);
 }
 
+// Split form (zh_pip.cuh): parity bitmaps of every pair, then the cells.
+#ifndef ZH_PAR_THREADS
+#define ZH_PAR_THREADS 128
+#endif
+#ifndef ZH_PAR_MINB
+#define ZH_PAR_MINB 12
+#endif
+template <bool kRep>
+__global__ void __launch_bounds__(ZH_PAR_THREADS, ZH_PAR_MINB) k_parity(PipP p) {
+  if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
+  extern __shared__ __align__(16) uint32_t sh[];
+  __shared__ LongQ lq;
+  parity_pair_body<kRep>(p, blockIdx.x, sh, &lq);
+}
+
+template <int kMode, bool kU64>
+__global__ void __launch_bounds__(kPipThreads, ZH_PIP_MINB) k_pip_cells(PipP p) {
+  if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
+  extern __shared__ __align__(16) uint32_t sh[];
+  pip_cells_body<kMode, kU64>(p, blockIdx.x, sh);
+}
+
 cudaError_t launch_pip(Ctx& c) { return launch_pip_list(c, c.d_isect.as<int2>(), c.n_isect, nullptr); }
+
 
 PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev) {
   PipP p;
@@ -60,6 +91,11 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev) {
   p.rc = bm_budget_words / p.wpr;
   if (p.rc < 1) p.rc = 1;
   if (p.rc > c.rp.T) p.rc = c.rp.T;
+  p.wpo = (c.rp.T + 31) / 32;
+  p.rcc = 8192 / p.wpo;
+  if (p.rcc < 1) p.rcc = 1;
+  if (p.rcc > c.rp.T) p.rcc = c.rp.T;
+  p.pbits = c.d_pbits.as<uint32_t>();
   return p;
 }
 
@@ -67,11 +103,63 @@ size_t pip_smem(const Ctx& c, const PipP& p) {
   return (size_t)hist_words(c.bp.nbins) * 4 + (size_t)p.rc * p.wpr * 4;
 }
 
+static cudaError_t launch_pip_fused_body(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
+
+static int pip_mode(const Ctx& c) {
+  const FastBins fb = make_fast_bins(c.bp);
+  return fast_bins_ok(c.bp) ? (fb.bias ? 4 : (c.bp.use_nodata ? 3 : 2)) : (c.bp.width == 1 ? 0 : 1);
+}
+
+cudaError_t pip_prepare(Ctx& c, int64_t grid) {
+  const size_t need = (size_t)grid * (size_t)c.rp.T * (size_t)((c.rp.T + 31) / 32) * 4;
+  return c.d_pbits.ensure(need);
+}
+
+cudaError_t launch_parity(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev, cudaStream_t s) {
+  if (grid == 0) return cudaSuccess;
+  PipP p = pip_params(c, pairs, n_dev);
+  const size_t smem = ((size_t)p.rc * p.wpr + 3) / 4 * 16;
+  const bool rep = !(c.geo.ox == 0.5 && c.geo.oy == 0.5);
+  void (*k)(PipP) = rep ? k_parity<true> : k_parity<false>;
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<(unsigned)grid, ZH_PAR_THREADS, smem, s>>>(p);
+  c.launches += 1;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pip_cells(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
+  if (grid == 0) return cudaSuccess;
+  PipP p = pip_params(c, pairs, n_dev);
+  const size_t smem = (size_t)hist_words(c.bp.nbins) * 4 + (size_t)p.rcc * p.wpo * 4;
+  void (*k)(PipP);
+  switch (pip_mode(c)) {
+    case 0: k = c.out_u64 ? k_pip_cells<0, true> : k_pip_cells<0, false>; break;
+    case 1: k = c.out_u64 ? k_pip_cells<1, true> : k_pip_cells<1, false>; break;
+    case 2: k = c.out_u64 ? k_pip_cells<2, true> : k_pip_cells<2, false>; break;
+    case 3: k = c.out_u64 ? k_pip_cells<3, true> : k_pip_cells<3, false>; break;
+    default: k = c.out_u64 ? k_pip_cells<4, true> : k_pip_cells<4, false>; break;
+  }
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<(unsigned)grid, kPipThreads, smem, c.stream>>>(p);
+  c.launches += 1;
+  return cudaGetLastError();
+}
+
 cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
+  if (grid == 0) return cudaSuccess;
+  if (c.pip_split) {
+    cudaError_t e = pip_prepare(c, grid);
+    if (e != cudaSuccess) return e;
+    if ((e = launch_parity(c, pairs, grid, n_dev, c.stream)) != cudaSuccess) return e;
+    return launch_pip_cells(c, pairs, grid, n_dev);
+  }
+  return launch_pip_fused_body(c, pairs, grid, n_dev);
+}
+
+static cudaError_t launch_pip_fused_body(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
   if (grid == 0) return cudaSuccess;
   PipP p = pip_params(c, pairs, n_dev);
   const size_t smem = pip_smem(c, p);
-  const int threads = 256;
   void (*k)(PipP);
   const int mode = fast_bins_ok(c.bp) ? (p.fb.bias ? 4 : (c.bp.use_nodata ? 3 : 2)) : (c.bp.width == 1 ? 0 : 1);
   const bool rep = !(c.geo.ox == 0.5 && c.geo.oy == 0.5);
@@ -86,7 +174,7 @@ cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64
   }
 #undef ZH_PIP_K
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k<<<(unsigned)grid, threads, smem, c.stream>>>(p);
+  k<<<(unsigned)grid, 256, smem, c.stream>>>(p);
   c.launches += 1;
   return cudaGetLastError();
 }

@@ -139,7 +139,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   c->rp.tr0 = (int32_t)tr0;
   c->rp.TRn = (int32_t)TRn;
   c->geo = zh::Geo{r->gt[0], r->gt[1], r->gt[3], r->gt[5], o->rep_custom ? o->rep_x : 0.5,
-                   o->rep_custom ? o->rep_y : 0.5};
+                   o->rep_custom ? o->rep_y : 0.5, 1.0 / r->gt[1]};
   c->on_host = r->on_host != 0;
   c->host_data = r->on_host ? r->data : nullptr;
   c->bp = zh::BinP{b->lo, b->width, b->nbins, b->use_nodata ? 1 : 0, b->nodata, b->oor_drop ? 1 : 0};
@@ -188,8 +188,12 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   }
   if ((e = cudaHostAlloc((void**)&c->pinned_counts, 8 * sizeof(int64_t), cudaHostAllocDefault)) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (pinned counters)"));
-  for (int i = 0; i < 13; ++i)
+  for (int i = 0; i < 16; ++i)
     if ((e = cudaEventCreate(&c->ev[i])) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (events)"));
+  if ((e = cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming)) != cudaSuccess)
+    return cleanup_fail(cuda_fail(e, "zh_create (side stream)"));
   if ((e = cudaGetLastError()) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
   *out = reinterpret_cast<zh_ctx>(c);
   return ZH_OK;
@@ -205,10 +209,16 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
-                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_fcounts, &c->d_stats};
+                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_fcounts, &c->d_stats};
   for (auto* b : bufs) b->release();
-  for (int i = 0; i < 13; ++i)
+  for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  if (c->side) {
+    cudaStreamSynchronize(c->side);
+    cudaStreamDestroy(c->side);
+  }
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->pinned_counts) cudaFreeHost(c->pinned_counts);
   delete c;
 }
@@ -220,7 +230,7 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
-                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_fcounts, &c.d_stats};
+                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_fcounts, &c.d_stats};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;
@@ -508,9 +518,10 @@ extern "C" zh_status zh_get_step_ms(zh_ctx h, float* ms, int32_t n) {
   Ctx* c = C(h);
   if (!c->timing) return fail(ZH_ERR_STATE, "timing is disabled");
   ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_step_ms");
-  // (start, stop) event pairs: steps 1..4, fused, fused pure-tile kernel, fused cell-in-polygon kernel
-  const int pairs[7][2] = {{0, 1}, {2, 3}, {4, 5}, {6, 7}, {8, 9}, {10, 11}, {11, 12}};
-  for (int i = 0; i < n && i < 7; ++i) {
+  // (start, stop) event pairs: steps 1..4, fused, fused pure-tile kernel, fused cell-in-polygon
+  // (cell) kernel, fused parity kernel (second stream, overlapping the pure-tile kernel)
+  const int pairs[8][2] = {{0, 1}, {2, 3}, {4, 5}, {6, 7}, {8, 9}, {10, 11}, {15, 12}, {13, 14}};
+  for (int i = 0; i < n && i < 8; ++i) {
     float v = 0.f;
     if (cudaEventElapsedTime(&v, c->ev[pairs[i][0]], c->ev[pairs[i][1]]) != cudaSuccess) {
       cudaGetLastError();

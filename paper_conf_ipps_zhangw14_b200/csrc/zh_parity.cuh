@@ -47,7 +47,7 @@ __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr,
   const int w = t.w;
   const double yc = row_centre<kRep>(g, r);
   const double xi = intercept(e, yc);
-  const double est = (xi - g.gt0) / g.gt1 - g.ox - (double)t.c0;
+  const double est = (xi - g.gt0) * g.igt1 - g.ox - (double)t.c0;
   int64_t ei;
   if (!(est > 0.0)) ei = 0;
   else if (est > (double)w) ei = w;
@@ -128,6 +128,37 @@ __device__ __forceinline__ void suffix_xor_rows(uint32_t* __restrict__ bm, int w
       t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
       row[wi] = (t >> 1) ^ (carry ? 0xFFFFFFFFu : 0u);
       carry ^= (t & 1u);
+    }
+  }
+}
+
+// Step 2 for the split form: rows [0, ch) of bm become parity bits written straight to `out`
+// (row stride wpo = ceil(w / 32) words, the word wpr - 1 = wpo only carries the "all cells" flips).
+// Thread per row; with wpo % 4 == 0 the row is produced 4 words at a time and stored as 16 bytes.
+__device__ __forceinline__ void suffix_xor_store(const uint32_t* __restrict__ bm, int wpr, int ch,
+                                                 uint32_t* __restrict__ out, int wpo) {
+  for (int lr = threadIdx.x; lr < ch; lr += blockDim.x) {
+    const uint32_t* row = bm + lr * wpr;
+    uint32_t* orow = out + (int64_t)lr * wpo;
+    uint32_t carry = 0;
+    auto step = [&](uint32_t t) -> uint32_t {
+      t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
+      const uint32_t v = (t >> 1) ^ (0u - carry);
+      carry ^= (t & 1u);
+      return v;
+    };
+    for (int wi = wpr - 1; wi >= wpo; --wi) step(row[wi]);
+    if ((wpo & 3) == 0) {
+      for (int g = wpo - 4; g >= 0; g -= 4) {
+        uint4 v;
+        v.w = step(row[g + 3]);
+        v.z = step(row[g + 2]);
+        v.y = step(row[g + 1]);
+        v.x = step(row[g]);
+        __stcs(reinterpret_cast<uint4*>(orow + g), v);
+      }
+    } else {
+      for (int wi = wpo - 1; wi >= 0; --wi) orow[wi] = step(row[wi]);
     }
   }
 }

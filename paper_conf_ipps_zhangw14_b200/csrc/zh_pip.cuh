@@ -1,5 +1,7 @@
 // zh_pip.cuh — step 4 for one (tile, polygon) pair, shared by k_pip and the fused kernel.
 #pragma once
+#include <type_traits>
+
 #include "zh_parity.cuh"
 
 namespace zh {
@@ -21,6 +23,9 @@ struct PipP {
   int wpr;  // bitmap words per row = T/32 + 1
   int rc;   // rows per chunk
   const int64_t* n_dev;  // device count of pairs (grid may be an upper bound), or nullptr
+  uint32_t* pbits;       // split form: per-pair parity bitmaps [pair][T][wpo] (global)
+  int wpo;               // words per stored parity row = ceil(T / 32)
+  int rcc;               // rows per chunk of the split cell kernel's shared copy of the bitmap
 };
 
 struct Ctx;  // zh_ctx.h
@@ -74,17 +79,25 @@ __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, u
     if (nk <= (int)blockDim.x) {
       const int rpi = blockDim.x / nk;
       const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
-      if (rs < rpi) {
+      // kA: the tile starts on a vector boundary (c0 % 8 == 0, e.g. T % 8 == 0), so each thread's 8
+      // parity bits are one byte of one bitmap word (no straddling)
+      auto run = [&](auto aligned) {
+        constexpr bool kA = decltype(aligned)::value;
         const int64_t cs = (k0 + kk) * 8;
         const uint32_t cskip = cols_skip8(cs, c0, w);
         const int lc0 = (int)(cs - c0);
+        const int wi = lc0 >> 5, bsh = lc0 & 31;
+        auto pbits = [&](int lr) -> uint32_t {
+          if (kA) return (bm[lr * p.wpr + wi] >> bsh) & 0xFFu;
+          return bits8(bm + lr * p.wpr, p.wpr, lc0);
+        };
         const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
         const int64_t step = (int64_t)rpi * pitch;
         int lr = rs;
         // two rows per iteration: both skip masks first, then both loads in flight
         for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
-          const uint32_t s0 = cskip | (~bits8(bm + lr * p.wpr, p.wpr, lc0) & 0xFFu);
-          const uint32_t s1 = cskip | (~bits8(bm + (lr + rpi) * p.wpr, p.wpr, lc0) & 0xFFu);
+          const uint32_t s0 = cskip | (~pbits(lr) & 0xFFu);
+          const uint32_t s1 = cskip | (~pbits(lr + rpi) & 0xFFu);
           uint4 q0 = make_uint4(0, 0, 0, 0), q1 = make_uint4(0, 0, 0, 0);
           if (s0 != 0xFFu) q0 = ld_stream16(ptr);
           if (s1 != 0xFFu) q1 = ld_stream16(ptr + step);
@@ -98,12 +111,16 @@ __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, u
           }
         }
         for (; lr < ch; lr += rpi, ptr += step) {
-          const uint32_t skip = cskip | (~bits8(bm + lr * p.wpr, p.wpr, lc0) & 0xFFu);
+          const uint32_t skip = cskip | (~pbits(lr) & 0xFFu);
           if (skip == 0xFFu) continue;
           const uint4 q = ld_stream16(ptr);
           if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q, skip, fb, dum2);
           else count8_generic<kMode == 0>(hist, q, skip, p.bp, dummy);
         }
+      };
+      if (rs < rpi) {
+        if ((c0 & 7) == 0) run(std::integral_constant<bool, true>{});
+        else run(std::integral_constant<bool, false>{});
       }
     } else {
       for (int lr = 0; lr < ch; ++lr) {
@@ -123,6 +140,147 @@ __device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, u
   const int nbins = p.bp.nbins;
   const int64_t orow = (int64_t)k * nbins;
   for (int b = threadIdx.x * 4; b < nbins; b += blockDim.x * 4) {  // 16-byte reads, zero vectors skipped
+    const uint4 v = *reinterpret_cast<const uint4*>(&hist[kOff + b]);
+    if (!(v.x | v.y | v.z | v.w)) continue;
+    const uint32_t vs[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (vs[q] && b + q < nbins) {
+        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(p.out) + orow + b + q, (unsigned long long)vs[q]);
+        else atomicAdd(reinterpret_cast<uint32_t*>(p.out) + orow + b + q, vs[q]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// Split form of the same step-4 work (the default): the parity phase of every pair runs in its own
+// kernel (k_parity, FP64-latency bound, run concurrently with the pure-tile kernel on a second
+// stream) and stores the pair's inside bits to HBM; the cell kernel (k_pip_cells) then streams each
+// pair's tile with no crossing phase and no barrier waiting on the slowest crossing thread.
+// ------------------------------------------------------------------------------------------------
+
+// Parity bits of pair `pair_idx` into p.pbits[pair_idx][r][0..wpo) (rows r < h of the tile).
+// `bm` holds rc * wpr words; `lq` as for pip_pair_body.
+template <bool kRep>
+__device__ __forceinline__ void parity_pair_body(const PipP& p, int64_t pair_idx, uint32_t* __restrict__ bm,
+                                                 LongQ* lq) {
+  if (threadIdx.x == 0) lq->n = 0;
+  const RasterP& rp = p.rp;
+  const Geo& g = p.g;
+  const int2 pr = p.isect[pair_idx];
+  const int tile = pr.x, k = pr.y;
+  const TileGeom t = tile_geom<kRep>(rp, g, tile);
+  const int64_t r0 = t.r0;
+  const int h = t.h;
+  const int4 m = p.mbb[k];
+  const int64_t band = p.band_base[k] + ((int)(r0 / rp.T) - m.z);
+  const int e0 = p.band_off[band], e1 = p.band_off[band + 1];
+  const int wpo = p.wpo, wpr = p.wpr;
+  uint32_t* __restrict__ out = p.pbits + pair_idx * (int64_t)rp.T * wpo;
+  for (int cr = 0; cr < h; cr += p.rc) {
+    const int ch = min(p.rc, h - cr);
+    const int64_t rlo = r0 + cr, rhi = rlo + ch;
+    for (int i = threadIdx.x * 4; i < ch * wpr; i += blockDim.x * 4)  // bm holds rc * wpr rounded up to 4
+      *reinterpret_cast<uint4*>(&bm[i]) = make_uint4(0, 0, 0, 0);
+    __syncthreads();
+    crossings_to_bitmap<kRep>(bm, wpr, e0, e1, p.band_edges, p.edges, p.erows, g, t, rlo, rhi, lq);
+    suffix_xor_store(bm, wpr, ch, out + (int64_t)cr * wpo, wpo);
+    __syncthreads();  // before the next chunk clears bm
+  }
+}
+
+// Cells of pair `pair_idx` with the parity bits of k_parity.  `sh` holds hist_words(nbins) +
+// rcc * wpo words.
+template <int kMode, bool kU64>
+__device__ __forceinline__ void pip_cells_body(const PipP& p, int64_t pair_idx, uint32_t* __restrict__ sh) {
+  const int HW = hist_words(p.bp.nbins);
+  uint32_t* hist = sh;
+  uint32_t* bm = sh + HW;
+  const RasterP& rp = p.rp;
+  const int2 pr = p.isect[pair_idx];
+  const int tile = pr.x, k = pr.y;
+  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int64_t r0 = (int64_t)(rp.tr0 + trl) * rp.T, c0 = (int64_t)tc * rp.T;
+  const int h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - r0);
+  const int w = (int)min((int64_t)rp.T, rp.cols - c0);
+  const int wpo = p.wpo;
+  const uint32_t* __restrict__ src = p.pbits + pair_idx * (int64_t)rp.T * wpo;
+
+  for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
+    *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
+  const uint32_t dummy = (uint32_t)hist_dummy(p.bp.nbins) + (threadIdx.x & 31);
+  const uint32_t dum2 = dummy * 0x10001u;
+  const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
+  const int nk = (int)(k1 - k0);
+  const int64_t pitch = rp.pitch;
+  const FastBins fb = p.fb;
+  auto count = [&](const uint4& q, uint32_t skip) {
+    if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q, skip, fb, dum2);
+    else count8_generic<kMode == 0>(hist, q, skip, p.bp, dummy);
+  };
+
+  for (int cr = 0; cr < h; cr += p.rcc) {
+    const int ch = min(p.rcc, h - cr);
+    const uint32_t* s = src + (int64_t)cr * wpo;
+    if ((wpo & 3) == 0) {
+      for (int i = threadIdx.x * 4; i < ch * wpo; i += blockDim.x * 4)
+        *reinterpret_cast<uint4*>(&bm[i]) = __ldcs(reinterpret_cast<const uint4*>(s + i));
+    } else {
+      for (int i = threadIdx.x; i < ch * wpo; i += blockDim.x) bm[i] = __ldcs(s + i);
+    }
+    __syncthreads();
+    const int16_t* base = rp.data + (r0 + cr - rp.row0) * pitch + k0 * 8;
+    if (nk <= (int)blockDim.x) {
+      const int rpi = blockDim.x / nk;
+      const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
+      auto run = [&](auto aligned) {
+        constexpr bool kA = decltype(aligned)::value;
+        const int64_t cs = (k0 + kk) * 8;
+        const uint32_t cskip = cols_skip8(cs, c0, w);
+        const int lc0 = (int)(cs - c0);
+        const int wi = lc0 >> 5, bsh = lc0 & 31;
+        auto pbits = [&](int lr) -> uint32_t {
+          if (kA) return (bm[lr * wpo + wi] >> bsh) & 0xFFu;
+          return bits8(bm + lr * wpo, wpo, lc0);
+        };
+        const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
+        const int64_t step = (int64_t)rpi * pitch;
+        int lr = rs;
+        for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
+          const uint32_t s0 = cskip | (~pbits(lr) & 0xFFu);
+          const uint32_t s1 = cskip | (~pbits(lr + rpi) & 0xFFu);
+          uint4 q0 = make_uint4(0, 0, 0, 0), q1 = make_uint4(0, 0, 0, 0);
+          if (s0 != 0xFFu) q0 = ld_stream16(ptr);
+          if (s1 != 0xFFu) q1 = ld_stream16(ptr + step);
+          if (s0 != 0xFFu) count(q0, s0);
+          if (s1 != 0xFFu) count(q1, s1);
+        }
+        for (; lr < ch; lr += rpi, ptr += step) {
+          const uint32_t skip = cskip | (~pbits(lr) & 0xFFu);
+          if (skip == 0xFFu) continue;
+          count(ld_stream16(ptr), skip);
+        }
+      };
+      if (rs < rpi) {
+        if ((c0 & 7) == 0) run(std::integral_constant<bool, true>{});
+        else run(std::integral_constant<bool, false>{});
+      }
+    } else {
+      for (int lr = 0; lr < ch; ++lr) {
+        for (int kk = threadIdx.x; kk < nk; kk += blockDim.x) {
+          const int64_t cs = (k0 + kk) * 8;
+          const uint32_t skip = cols_skip8(cs, c0, w) | (~bits8(bm + lr * wpo, wpo, (int)(cs - c0)) & 0xFFu);
+          if (skip == 0xFFu) continue;
+          count(ld_stream16(base + (int64_t)lr * pitch + kk * 8), skip);
+        }
+      }
+    }
+    __syncthreads();
+  }
+  const int nbins = p.bp.nbins;
+  const int64_t orow = (int64_t)k * nbins;
+  for (int b = threadIdx.x * 4; b < nbins; b += blockDim.x * 4) {
     const uint4 v = *reinterpret_cast<const uint4*>(&hist[kOff + b]);
     if (!(v.x | v.y | v.z | v.w)) continue;
     const uint32_t vs[4] = {v.x, v.y, v.z, v.w};

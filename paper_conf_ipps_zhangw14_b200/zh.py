@@ -317,12 +317,12 @@ class ZonalHistogram:
         _check(LIB.zh_set_timing(self.h, int(enable)))
 
     STEP_NAMES = ("step1_tile_hist", "step2_pair_tiles", "step3_aggregate", "step4_pip_update", "fused_update",
-                  "fused_pure_kernel", "fused_pip_kernel")
+                  "fused_pure_kernel", "fused_pip_kernel", "fused_parity_kernel")
 
     def step_ms(self) -> dict:
         """Device ms of the last call of each step (-1: not called since timing was enabled)."""
-        ms = (ctypes.c_float * 7)()
-        _check(LIB.zh_get_step_ms(self.h, ms, 7))
+        ms = (ctypes.c_float * len(self.STEP_NAMES))()
+        _check(LIB.zh_get_step_ms(self.h, ms, len(self.STEP_NAMES)))
         return dict(zip(self.STEP_NAMES, list(ms)))
 
     def launch_count(self) -> int:
