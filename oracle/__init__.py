@@ -65,6 +65,13 @@ def _L():
         lib.zho_o1.restype = None
         lib.zho_o1.argtypes = [vp, i64, i64, i64, i64, i64, vp, i64, vp, vp, vp, vp, ctypes.POINTER(Bins), vp,
                                ctypes.c_int]
+        lib.zho_seg_touches.restype = ctypes.c_int
+        lib.zho_seg_touches.argtypes = [dbl] * 8
+        lib.zho_cover_o0.restype = None
+        lib.zho_cover_o0.argtypes = [vp, i64, i64, i64, i64, i64, vp, i64, vp, vp, vp, vp, ctypes.POINTER(Bins), vp,
+                                     ctypes.c_int, ctypes.c_int]
+        lib.zho_cover_membership.restype = None
+        lib.zho_cover_membership.argtypes = [vp, vp, i64, vp, i64, vp, vp, vp, vp, vp, ctypes.c_int]
         lib.zho_membership.restype = None
         lib.zho_membership.argtypes = [vp, vp, i64, vp, i64, vp, vp, vp, vp, vp, ctypes.c_int]
         _lib = lib
@@ -134,6 +141,30 @@ def o0(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, prefilter: bool = F
 def o1(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, nthreads=None, rep=None):
     """O1: row-hoisted intercepts, identical comparisons to O0.  Returns uint64 [n_poly, nbins]."""
     return _hist(_L().zho_o1, win, row0, col0, gt, P, bins, nthreads, (), rep)
+
+
+def seg_touches(x0, y0, x1, y1, X0, X1, Y0, Y1) -> bool:
+    """R15: does the segment (x0,y0)-(x1,y1) meet the closed rectangle between the grid lines?"""
+    return bool(_L().zho_seg_touches(*(float(v) for v in (x0, y0, x1, y1, X0, X1, Y0, Y1))))
+
+
+def cover_o0(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, prefilter: bool = True, nthreads=None):
+    """The "geometrically intersect" variant (reading R15): a cell counts in P_k when
+    its closed rectangle meets the closed polygon.  Returns uint64 [n_poly, nbins]."""
+    return _hist(_L().zho_cover_o0, win, row0, col0, gt, P, bins, nthreads, (int(prefilter),))
+
+
+def cover_membership(rows, cols, gt, P, nthreads=None) -> np.ndarray:
+    """covered[q, k] in {0,1} for the cells (rows[q], cols[q]) (reading R15)."""
+    rows = _c64(rows, np.int64)
+    cols = _c64(cols, np.int64)
+    g = _gt8(gt)
+    pro, rvo, x, y = _poly_args(P)
+    out = np.zeros((rows.shape[0], P.n_poly), dtype=np.uint8)
+    _L().zho_cover_membership(rows.ctypes.data, cols.ctypes.data, rows.shape[0], g.ctypes.data, P.n_poly,
+                              pro.ctypes.data, rvo.ctypes.data, x.ctypes.data, y.ctypes.data, out.ctypes.data,
+                              _nthreads(nthreads))
+    return out
 
 
 def membership(rows, cols, gt, P, nthreads=None, rep=None) -> np.ndarray:

@@ -37,6 +37,10 @@
  *                      in increasing xc; a cell is inside iff #{xi > xc} is odd.  It evaluates
  *                      exactly the same (xc < xi) comparisons as O0, only once per
  *                      (edge,row) instead of once per (edge,cell).  Pinned O0 == O1.
+ *   zho_seg_touches    R15: does a segment meet a closed cell rectangle (separating-axis test)
+ *   zho_cover_o0       the "geometrically intersect" variant: a cell counts in P_k
+ *                      when its closed rectangle meets the closed polygon — its centre is inside
+ *                      (the test above) or some edge of P_k meets the rectangle (end of file)
  */
 #include <math.h>
 #include <stdint.h>
@@ -257,4 +261,103 @@ void zho_membership(const int64_t* rows, const int64_t* cols, int64_t nq, const 
     for (int64_t k = 0; k < n_poly; ++k)
       inside[q * n_poly + k] = (uint8_t)(zho_crossings(xc, yc, k, pro, rvo, x, y) & 1);
   }
+}
+
+/* ---------------------------------------------------------------------------------------------
+ * Reading R15 — the literal "cells that geometrically intersect with P_k" (§III ¶1;
+ * the paper then picks the cell centre, §III.D).  A cell (r, c) is the CLOSED
+ * rectangle between the grid lines X(c), X(c+1) and Y(r), Y(r+1), with
+ *     X(c) = gt0 + (double)c * gt1,   Y(r) = gt3 + (double)r * gt5   (two IEEE ops each, no FMA).
+ * It meets the closed region of P_k iff its centre is inside P_k (the crossing test above, which
+ * decides the cells no edge reaches) or some edge of P_k meets the rectangle.  Segment vs closed
+ * rectangle is the separating-axis test: the bounding boxes overlap (closed comparisons) and the
+ * four corners are not all strictly on one side of the segment's line, with the orientation
+ *     o(P) = dx * (Py - ya) - dy * (Px - xa),   dx = xb - xa,  dy = yb - ya,
+ * each product and difference one binary64 op, the endpoints ordered lexicographically by (y, x)
+ * so that the result depends on the undirected segment only.  A segment that only touches the
+ * rectangle (a corner or a side) meets it: the sets are closed (ST_Intersects semantics).
+ * --------------------------------------------------------------------------------------------- */
+static inline double grid_x(const double* gt, int64_t c) { double t = (double)c * gt[1]; return gt[0] + t; }
+static inline double grid_y(const double* gt, int64_t r) { double t = (double)r * gt[5]; return gt[3] + t; }
+
+int zho_seg_touches(double x0, double y0, double x1, double y1, double X0, double X1, double Y0, double Y1) {
+  const double xlo = X0 < X1 ? X0 : X1, xhi = X0 < X1 ? X1 : X0;
+  const double ylo = Y0 < Y1 ? Y0 : Y1, yhi = Y0 < Y1 ? Y1 : Y0;
+  if ((x0 > x1 ? x0 : x1) < xlo || (x0 < x1 ? x0 : x1) > xhi) return 0;
+  if ((y0 > y1 ? y0 : y1) < ylo || (y0 < y1 ? y0 : y1) > yhi) return 0;
+  double xa = x0, ya = y0, xb = x1, yb = y1;
+  if (ya > yb || (ya == yb && xa > xb)) { xa = x1; ya = y1; xb = x0; yb = y0; }
+  const double dx = xb - xa, dy = yb - ya;
+  const double cx[4] = {xlo, xhi, xlo, xhi}, cy[4] = {ylo, ylo, yhi, yhi};
+  int pos = 0, neg = 0;
+  for (int i = 0; i < 4; ++i) {
+    double u = cy[i] - ya;
+    double v = cx[i] - xa;
+    double p = dx * u;
+    double q = dy * v;
+    double o = p - q;
+    pos += o > 0;
+    neg += o < 0;
+  }
+  return !(pos == 4 || neg == 4);
+}
+
+/* Does polygon k meet the closed rectangle of cell (r, c)? */
+static int cell_covered(const double* gt, int64_t r, int64_t c, int64_t k, const int64_t* pro, const int64_t* rvo,
+                        const double* x, const double* y) {
+  double xc, yc;
+  zho_centre(gt, r, c, &xc, &yc);
+  if (zho_crossings(xc, yc, k, pro, rvo, x, y) & 1) return 1;
+  const double X0 = grid_x(gt, c), X1 = grid_x(gt, c + 1), Y0 = grid_y(gt, r), Y1 = grid_y(gt, r + 1);
+  for (int64_t rg = pro[k]; rg < pro[k + 1]; ++rg) {
+    int64_t a = rvo[rg], m = rvo[rg + 1] - a;
+    for (int64_t e = 0; e < m; ++e) {
+      int64_t f = (e + 1 == m) ? 0 : e + 1;
+      if (zho_seg_touches(x[a + e], y[a + e], x[a + f], y[a + f], X0, X1, Y0, Y1)) return 1;
+    }
+  }
+  return 0;
+}
+
+/* The cover variant of O0 (gt[6], gt[7] must be 0.5: the centre decides the cells no edge reaches).
+ * prefilter = 1 skips polygon k at a cell whose closed rectangle misses k's closed vertex bounding
+ * box: then no edge meets it, and the centre, half a cell outside the box, is outside (the O0
+ * prefilter argument) — pinned against prefilter = 0. */
+void zho_cover_o0(const int16_t* win, int64_t row0, int64_t col0, int64_t nrows, int64_t ncols, int64_t pitch,
+                  const double* gt, int64_t n_poly, const int64_t* pro, const int64_t* rvo, const double* x,
+                  const double* y, const zho_bins* bins, uint64_t* out, int prefilter, int nthreads) {
+  bbox_t* bb = (bbox_t*)malloc(sizeof(bbox_t) * (size_t)(n_poly > 0 ? n_poly : 1));
+  for (int64_t k = 0; k < n_poly; ++k) poly_bbox(k, pro, rvo, x, y, &bb[k]);
+  if (nthreads < 1) nthreads = 1;
+#pragma omp parallel for schedule(dynamic, 1) num_threads(nthreads)
+  for (int64_t i = 0; i < nrows; ++i) {
+    for (int64_t j = 0; j < ncols; ++j) {
+      int b = zho_bin(win[i * pitch + j], bins);
+      if (b < 0) continue;
+      const int64_t r = row0 + i, c = col0 + j;
+      const double X0 = grid_x(gt, c), X1 = grid_x(gt, c + 1), Y0 = grid_y(gt, r), Y1 = grid_y(gt, r + 1);
+      const double xlo = X0 < X1 ? X0 : X1, xhi = X0 < X1 ? X1 : X0;
+      const double ylo = Y0 < Y1 ? Y0 : Y1, yhi = Y0 < Y1 ? Y1 : Y0;
+      for (int64_t k = 0; k < n_poly; ++k) {
+        if (prefilter) {
+          if (bb[k].empty) continue;
+          if (xhi < bb[k].xmin || xlo > bb[k].xmax || yhi < bb[k].ymin || ylo > bb[k].ymax) continue;
+        }
+        if (cell_covered(gt, r, c, k, pro, rvo, x, y))
+          __atomic_fetch_add(&out[k * bins->nbins + b], (uint64_t)1, __ATOMIC_RELAXED);
+      }
+    }
+  }
+  free(bb);
+}
+
+/* Per-cell cover membership for a list of cells: covered[q*n_poly + k] in {0,1}. */
+void zho_cover_membership(const int64_t* rows, const int64_t* cols, int64_t nq, const double* gt, int64_t n_poly,
+                          const int64_t* pro, const int64_t* rvo, const double* x, const double* y,
+                          uint8_t* covered, int nthreads) {
+  if (nthreads < 1) nthreads = 1;
+#pragma omp parallel for schedule(dynamic, 16) num_threads(nthreads)
+  for (int64_t q = 0; q < nq; ++q)
+    for (int64_t k = 0; k < n_poly; ++k)
+      covered[q * n_poly + k] = (uint8_t)cell_covered(gt, rows[q], cols[q], k, pro, rvo, x, y);
 }

@@ -62,7 +62,10 @@ __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr,
 // Shared-memory queue of long edges (more than kLongRows straddled rows in the chunk): they are
 // processed afterwards by whole warps, one row per lane, so that no thread serialises hundreds of
 // rows while the others wait at the barrier.
-constexpr int kLongRows = 8;
+#ifndef ZH_LONG_ROWS
+#define ZH_LONG_ROWS 8
+#endif
+constexpr int kLongRows = ZH_LONG_ROWS;
 constexpr int kLongQ = 128;
 struct LongQ {
   int n;
