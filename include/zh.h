@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 3
+#define ZH_ABI_VERSION 4
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -122,7 +122,11 @@ typedef struct {
                           1: the point (c + rep_x, r + rep_y) in cell units, rep_x, rep_y in
                           [0, 1] — e.g. (0, 0) the cell corner at the origin of the cell
                           (the alternatives of PAPER.md:18)                   */
-  int32_t reserved;
+  int32_t cover;       /* 0: a cell counts in P_k when its representative point is inside (the
+                          paper's choice, §III.D); 1: when its CLOSED rectangle meets
+                          the CLOSED polygon — the literal "cells that geometrically intersect
+                          with P_k" of PAPER.md:12 §III ¶1 (R15; touching counts).
+                          Requires rep_custom = 0 (ZH_ERR_UNSUPPORTED otherwise)               */
   double rep_x, rep_y;
 } zh_options;
 

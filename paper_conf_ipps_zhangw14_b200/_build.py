@@ -8,7 +8,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libzh.so")
-SOURCES = ["zh_api.cu", "k_tile_hist.cu", "k_pairs.cu", "k_aggregate.cu", "k_pip.cu", "k_fused.cu", "k_stats.cu"]
+SOURCES = ["zh_api.cu", "k_tile_hist.cu", "k_pairs.cu", "k_aggregate.cu", "k_pip.cu", "k_fused.cu", "k_stats.cu", "k_touch.cu"]
 HEADERS = ["zh_internal.cuh", "zh_ctx.h", "zh_tilehist.cuh", "zh_parity.cuh", "zh_pip.cuh"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",

@@ -95,7 +95,7 @@ __global__ void k_pure_tiles(const uint32_t* __restrict__ pure_cnt, int64_t n, c
 __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, const int2* __restrict__ inside,
                            int64_t n_inside, const uint32_t* __restrict__ extra, const uint32_t* __restrict__ pip_off,
                            uint32_t* __restrict__ cursor, int64_t n_tiles, RasterP rp, int2* __restrict__ pip,
-                           int64_t* __restrict__ counts) {
+                           int32_t* __restrict__ remap, int64_t* __restrict__ counts) {
   const int64_t n = n_isect + n_inside;
   int64_t cells = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
@@ -106,7 +106,9 @@ __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, cons
       if (!extra[i - n_isect]) continue;
       pr = inside[i - n_isect];
     }
-    pip[pip_off[pr.x] + atomicAdd(&cursor[pr.x], 1u)] = pr;
+    const uint32_t pos = pip_off[pr.x] + atomicAdd(&cursor[pr.x], 1u);
+    pip[pos] = pr;
+    if (remap && i < n_isect) remap[i] = (int32_t)pos;  // isect index -> list index (k_touch)
     cells += tile_cells(rp, pr.x);
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) counts[1] = (int64_t)pip_off[n_tiles];
@@ -249,6 +251,7 @@ cudaError_t launch_fused(Ctx& c) {
   if ((e = c.d_extra_pos.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pip.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
   if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 4)) != cudaSuccess) return e;
+  if (c.cover && (e = c.d_remap.ensure(sizeof(int32_t) * ((size_t)NX + 1))) != cudaSuccess) return e;
   cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 4, c.stream);
   if (NT == 0 || NI + NX == 0) {
     if (c.timing)
@@ -288,6 +291,7 @@ cudaError_t launch_fused(Ctx& c) {
   k_pip_list<<<grid_for(NI + NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_inside.as<int2>(), NI,
                                                           c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(),
                                                           c.d_pip_cur.as<uint32_t>(), NT, c.rp, c.d_pip.as<int2>(),
+                                                          c.cover ? c.d_remap.as<int32_t>() : nullptr,
                                                           c.d_fcounts.as<int64_t>());
   c.launches += 1;
 
@@ -296,7 +300,7 @@ cudaError_t launch_fused(Ctx& c) {
   // mixed tiles, split form: the parity bitmaps of every cell-in-polygon pair are built on the side
   // stream WHILE the pure-tile kernel streams the pure tiles (FP64-latency work beside HBM-bound
   // work), then the cell kernel runs once both are done
-  const bool split = c.pip_split != 0;
+  const bool split = c.pip_split != 0 || c.cover != 0;
   if (split) {
     if ((e = pip_prepare(c, NI + NX)) != cudaSuccess) return e;
     cudaEventRecord(c.ev_fork, c.stream);
@@ -305,6 +309,9 @@ cudaError_t launch_fused(Ctx& c) {
     if ((e = launch_parity(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1,
                            ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess)
       return e;
+    if (c.cover) {  // R15: cells an edge reaches join the parity bits (k_touch.cu)
+      if ((e = launch_touch(c, c.d_remap.as<int32_t>(), ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess) return e;
+    }
     if (c.timing) cudaEventRecord(c.ev[14], ZH_PAR_SIDE ? c.side : c.stream);
     cudaEventRecord(c.ev_join, c.side);
   }

@@ -147,10 +147,11 @@ cudaError_t launch_pip_cells(Ctx& c, const int2* pairs, int64_t grid, const int6
 
 cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
   if (grid == 0) return cudaSuccess;
-  if (c.pip_split) {
+  if (c.pip_split || c.cover) {
     cudaError_t e = pip_prepare(c, grid);
     if (e != cudaSuccess) return e;
     if ((e = launch_parity(c, pairs, grid, n_dev, c.stream)) != cudaSuccess) return e;
+    if (c.cover && pairs == c.d_isect.as<int2>() && (e = launch_touch(c, nullptr, c.stream)) != cudaSuccess) return e;
     return launch_pip_cells(c, pairs, grid, n_dev);
   }
   return launch_pip_fused_body(c, pairs, grid, n_dev);

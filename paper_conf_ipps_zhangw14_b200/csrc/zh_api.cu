@@ -54,6 +54,9 @@ static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bin
   if (o->tile < 1) return fail(ZH_ERR_INVALID_ARG, "tile must be >= 1");
   if (o->rep_custom && !(o->rep_x >= 0.0 && o->rep_x <= 1.0 && o->rep_y >= 0.0 && o->rep_y <= 1.0))
     return fail(ZH_ERR_INVALID_ARG, "representative point offsets must lie in [0, 1]");
+  if (o->cover != 0 && o->cover != 1) return fail(ZH_ERR_INVALID_ARG, "cover must be 0 or 1");
+  if (o->cover && o->rep_custom)
+    return fail(ZH_ERR_UNSUPPORTED, "cover mode decides the cells no edge reaches by their centre (rep_custom = 0)");
   if (r->row0 % o->tile != 0) return fail(ZH_ERR_INVALID_ARG, "row0 must be a multiple of the tile size");
   for (int i = 0; i < 6; ++i)
     if (!isfinite(r->gt[i])) return fail(ZH_ERR_INVALID_ARG, "geotransform must be finite");
@@ -146,6 +149,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   c->B_pad = (b->nbins + 3) & ~3;
   c->out_u64 = o->out_u64 ? 1 : 0;
   c->force_isect = o->force_isect ? 1 : 0;
+  c->cover = o->cover ? 1 : 0;
   c->fused = o->fused ? 1 : 0;
   c->stream = (cudaStream_t)o->stream;
   c->n_tiles = n_tiles;
@@ -209,7 +213,7 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
-                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_fcounts, &c->d_stats};
+                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats};
   for (auto* b : bufs) b->release();
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
@@ -230,7 +234,7 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
-                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_fcounts, &c.d_stats};
+                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;

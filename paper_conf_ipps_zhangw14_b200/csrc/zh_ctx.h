@@ -48,6 +48,7 @@ struct Ctx {
   int32_t B_pad = 0;
   int32_t out_u64 = 1;
   int32_t force_isect = 0;
+  int32_t cover = 0;  // R15: closed cell rectangle meets the closed polygon (k_touch.cu)
   int32_t pip_split = ZH_PIP_SPLIT_DEFAULT;  // step 4 as k_parity + k_pip_cells (1) or one k_pip kernel per pair (0)
   cudaStream_t stream = nullptr;
   // polygons (device)
@@ -59,7 +60,7 @@ struct Ctx {
   DBuf d_inside, d_isect, d_counts, d_cub;
   // fused path lists (k_fused.cu)
   DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,
-      d_pip, d_pip_cur, d_fcounts, d_pbits;
+      d_pip, d_pip_cur, d_fcounts, d_pbits, d_remap;
   DBuf d_stats;  // zonal statistics [P][8] (k_stats.cu)
   int64_t n_cand = 0, n_bands = 0, n_band_entries = 0, n_inside = 0, n_isect = 0;
   // step 1 product and output
@@ -91,6 +92,7 @@ cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64
 cudaError_t pip_prepare(Ctx& c, int64_t grid);  // split form: per-pair parity bitmap buffer
 cudaError_t launch_parity(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev, cudaStream_t s);
 cudaError_t launch_pip_cells(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
+cudaError_t launch_touch(Ctx& c, const int32_t* remap, cudaStream_t s);  // k_touch.cu (cover mode)
 cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
 cudaError_t launch_zonal_stats(Ctx& c, int64_t* dstats);  // k_stats.cu
 cudaError_t launch_row_cost(Ctx& c, double* d_row_cost);  // k_fused.cu (shard planning)

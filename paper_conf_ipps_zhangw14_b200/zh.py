@@ -50,7 +50,7 @@ class zh_bins(ctypes.Structure):
 class zh_options(ctypes.Structure):
     _fields_ = [("tile", ctypes.c_int32), ("out_u64", ctypes.c_int32), ("force_isect", ctypes.c_int32),
                 ("fused", ctypes.c_int32), ("stream", ctypes.c_void_p), ("rep_custom", ctypes.c_int32),
-                ("reserved", ctypes.c_int32), ("rep_x", ctypes.c_double), ("rep_y", ctypes.c_double)]
+                ("cover", ctypes.c_int32), ("rep_x", ctypes.c_double), ("rep_y", ctypes.c_double)]
 
 
 class zh_stats(ctypes.Structure):
@@ -167,12 +167,14 @@ class ZonalHistogram:
     row `row0` of a raster with `rows` rows (default: a single shard holding the whole raster).
     polygons: any object with poly_ring_off, ring_vert_off, x, y arrays (synth.polygons.Polygons).
     rep: None for cell centres, or (ox, oy) in [0, 1]^2 — the representative point (c+ox, r+oy).
+    cover: count a cell in P_k when its closed rectangle meets the closed polygon (the literal
+    "geometrically intersect" of PAPER.md:12; R15) instead of testing its centre.
     """
 
     def __init__(self, raster, gt, polygons, nbins: int, lo: int = 0, width: int = 1, nodata=None,
                  oor_drop: bool = False, tile: int = 256, out_u64: bool = True, force_isect: bool = False,
                  row0: int = 0, rows: int | None = None, cols: int | None = None, stream=None,
-                 fused: bool = True, rep=None):
+                 fused: bool = True, rep=None, cover: bool = False):
         self._keep = []
         on_host, ptr, nrows, ncols_buf, pitch = self._raster_ptr(raster)
         ncols = cols if cols is not None else ncols_buf
@@ -194,7 +196,7 @@ class ZonalHistogram:
         b = zh_bins(lo, width, nbins, 0 if nodata is None else 1, 0 if nodata is None else int(nodata), int(oor_drop))
         self.stream = _stream_handle(stream)
         o = zh_options(tile, int(out_u64), int(force_isect), int(fused), self.stream,
-                       0 if rep is None else 1, 0, 0.5 if rep is None else float(rep[0]),
+                       0 if rep is None else 1, int(cover), 0.5 if rep is None else float(rep[0]),
                        0.5 if rep is None else float(rep[1]))
         h = ctypes.c_void_p()
         _check(LIB.zh_create(ctypes.byref(h), ctypes.byref(r), ctypes.byref(p), ctypes.byref(b), ctypes.byref(o)))
