@@ -205,6 +205,9 @@ def main():
     ap.add_argument("--path", default="fused", choices=["fused", "four_step"],
                     help="fused: step 2 + zh_fused_update (steps 1+3+4 fused, SURVEY §8f-1); four_step: 2,1,3,4")
     ap.add_argument("--no-other", action="store_true", help="skip timing the other path")
+    ap.add_argument("--cover", action="store_true",
+                    help="count cells whose closed rectangle meets the polygon (R15, PAPER.md:12) instead of "
+                         "testing the cell centre (not the headline configuration)")
     ap.add_argument("--equal-shards", action="store_true",
                     help="N > 1: equal tile-row strips instead of the work-balanced plan (zh_plan_rows)")
     args = ap.parse_args()
@@ -261,7 +264,7 @@ def main():
     out = torch.zeros((P.n_poly, cfg.nbins), dtype=torch.int64, device="cuda")
     z = zh.ZonalHistogram(raster_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
                           oor_drop=cfg.oor_drop, tile=T, rows=cfg.rows, cols=cfg.cols, row0=r0, stream=stream,
-                          fused=(args.path == "fused"))
+                          fused=(args.path == "fused"), cover=args.cover)
     z.set_output(out)
 
     path = args.path
@@ -405,7 +408,8 @@ def main():
                 "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert,
                                parallelism=f"tile-row shards x{world}" + (" (shared GPU, gloo)" if shared else "")
                                + ("" if world == 1 else (" equal" if args.equal_shards else " work-balanced")),
-                               l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA"),
+                               l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA",
+                               cells="closed rectangle meets polygon (R15)" if args.cover else "centre inside"),
                 "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
                 "clocks": clocks, "path": path, "steps_detail": steps_detail, "other_path": other,
                 "pairs": {k: st[k] for k in ("n_tiles", "n_candidates", "n_inside", "n_isect", "n_band_entries",
@@ -447,7 +451,7 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
         t0 = time.perf_counter()
         z2 = zh.ZonalHistogram(host_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
                                oor_drop=cfg.oor_drop, tile=cfg.tile, rows=cfg.rows, cols=cfg.cols, row0=r0,
-                               stream=stream, fused=(args.path == "fused"))
+                               stream=stream, fused=(args.path == "fused"), cover=args.cover)
         if world > 1:
             z2.set_output(out)
             z2.zh_run(None)

@@ -56,6 +56,7 @@ struct TouchP {
   const int32_t* remap;      // isect index -> index in the pair list of k_parity (nullptr: identity)
   uint32_t* pbits;           // [pair][T][wpo]
   int wpo;
+  double igt1, igt5;         // 1/gt1, 1/gt5 (candidate ranges only)
 };
 
 // Mark cell (r, c) of polygon k as covered in its pair's bitmap.
@@ -71,12 +72,18 @@ __device__ __forceinline__ void mark_cell(const TouchP& p, int k, const int4& m,
   atomicOr(&p.pbits[pi * (int64_t)T * p.wpo + (int64_t)lr * p.wpo + (lc >> 5)], 1u << (lc & 31));
 }
 
-// Cells of slab i (a row when kRows, else a column) that the segment meets: the minor-axis range
-// from the segment clipped to the slab, +-1 cell, each candidate decided exactly.
+// Candidate cell indices [ceil(q0 - d) - 1, floor(q1 + d)] along an axis for a real-valued index
+// interval [q0, q1]: cell j spans [j, j + 1] in index units, and it can meet the interval only if
+// j <= q1 and j + 1 >= q0.  d = 1e-3 cell absorbs the rounding of the (approximate) guesses; the
+// exact test decides every candidate.
+constexpr double kSlack = 1e-3;
+
+// Cells of slab i (a row when `rows`, else a column) that the segment meets: the minor-axis range
+// of the segment clipped to the slab (approximate: reciprocals, no exact arithmetic needed for a
+// candidate range), then the exact test for each candidate cell.
 __device__ __forceinline__ void touch_slab(const TouchP& p, int k, const int4& m, const Edge& e, bool rows,
-                                           int64_t i, int64_t lo2, int64_t hi2) {
+                                           int64_t i, int64_t lo2, int64_t hi2, double inv_da) {
   const Geo& g = p.g;
-  // slab extent along the major axis (as the same grid-line expressions the exact test uses)
   const double s0 = rows ? grid_y(g, i) : grid_x(g, i), s1 = rows ? grid_y(g, i + 1) : grid_x(g, i + 1);
   const double slo = fmin(s0, s1), shi = fmax(s0, s1);
   const double a0 = rows ? e.ya : e.xa, a1 = rows ? e.yb : e.xb;  // major coordinates of the ends
@@ -86,18 +93,15 @@ __device__ __forceinline__ void touch_slab(const TouchP& p, int k, const int4& m
     bmin = fmin(b0, b1);
     bmax = fmax(b0, b1);
   } else {
-    double t0 = (slo - a0) / (a1 - a0), t1 = (shi - a0) / (a1 - a0);
-    t0 = fmin(fmax(t0, 0.0), 1.0);
-    t1 = fmin(fmax(t1, 0.0), 1.0);
+    const double t0 = fmin(fmax((slo - a0) * inv_da, 0.0), 1.0), t1 = fmin(fmax((shi - a0) * inv_da, 0.0), 1.0);
     const double u0 = b0 + t0 * (b1 - b0), u1 = b0 + t1 * (b1 - b0);
     bmin = fmin(u0, u1);
     bmax = fmax(u0, u1);
   }
-  // minor-axis cell indices (real-valued), 1 cell of margin
-  double q0 = rows ? (bmin - g.gt0) / g.gt1 : (bmin - g.gt3) / g.gt5;
-  double q1 = rows ? (bmax - g.gt0) / g.gt1 : (bmax - g.gt3) / g.gt5;
+  double q0 = rows ? (bmin - g.gt0) * p.igt1 : (bmin - g.gt3) * p.igt5;
+  double q1 = rows ? (bmax - g.gt0) * p.igt1 : (bmax - g.gt3) * p.igt5;
   if (q0 > q1) { const double t = q0; q0 = q1; q1 = t; }
-  const double jlo = fmax(floor(q0) - 1.0, (double)lo2), jhi = fmin(floor(q1) + 1.0, (double)hi2);
+  const double jlo = fmax(ceil(q0 - kSlack) - 1.0, (double)lo2), jhi = fmin(floor(q1 + kSlack), (double)hi2);
   if (!(jlo <= jhi)) return;
   for (int64_t j = (int64_t)jlo; j <= (int64_t)jhi; ++j) {
     const int64_t r = rows ? i : j, c = rows ? j : i;
@@ -108,20 +112,22 @@ __device__ __forceinline__ void touch_slab(const TouchP& p, int k, const int4& m
 
 // Major axis and slab range of an edge (clipped to the shard rows / raster columns); false if empty.
 __device__ __forceinline__ bool edge_slabs(const TouchP& p, const Edge& e, bool& rows, int64_t& i0, int64_t& i1,
-                                           int64_t& lo2, int64_t& hi2) {
+                                           int64_t& lo2, int64_t& hi2, double& inv_da) {
   const Geo& g = p.g;
   const RasterP& rp = p.rp;
-  double ca = (fmin(e.xa, e.xb) - g.gt0) / g.gt1, cb = (fmax(e.xa, e.xb) - g.gt0) / g.gt1;
+  double ca = (fmin(e.xa, e.xb) - g.gt0) * p.igt1, cb = (fmax(e.xa, e.xb) - g.gt0) * p.igt1;
   if (ca > cb) { const double t = ca; ca = cb; cb = t; }
-  double ra = (e.ya - g.gt3) / g.gt5, rb = (e.yb - g.gt3) / g.gt5;
+  double ra = (e.ya - g.gt3) * p.igt5, rb = (e.yb - g.gt3) * p.igt5;
   if (ra > rb) { const double t = ra; ra = rb; rb = t; }
   const double R0 = (double)rp.row0, R1 = (double)(rp.row0 + rp.nrows - 1), C1 = (double)(rp.cols - 1);
-  const double rlo = fmax(floor(ra) - 1.0, R0), rhi = fmin(floor(rb) + 1.0, R1);
-  const double clo = fmax(floor(ca) - 1.0, 0.0), chi = fmin(floor(cb) + 1.0, C1);
+  const double rlo = fmax(ceil(ra - kSlack) - 1.0, R0), rhi = fmin(floor(rb + kSlack), R1);
+  const double clo = fmax(ceil(ca - kSlack) - 1.0, 0.0), chi = fmin(floor(cb + kSlack), C1);
   if (!(rlo <= rhi) || !(clo <= chi)) return false;
   rows = (rb - ra) >= (cb - ca);
   if (rows) { i0 = (int64_t)rlo; i1 = (int64_t)rhi; lo2 = 0; hi2 = rp.cols - 1; }
   else      { i0 = (int64_t)clo; i1 = (int64_t)chi; lo2 = rp.row0; hi2 = rp.row0 + rp.nrows - 1; }
+  const double da = rows ? e.yb - e.ya : e.xb - e.xa;
+  inv_da = da != 0.0 ? 1.0 / da : 0.0;
   return true;
 }
 
@@ -141,7 +147,8 @@ __global__ void __launch_bounds__(256) k_touch(TouchP p) {
     const Edge e = p.edges[v];
     bool rows;
     int64_t i0, i1, lo2, hi2;
-    if (!edge_slabs(p, e, rows, i0, i1, lo2, hi2)) continue;
+    double ida;
+    if (!edge_slabs(p, e, rows, i0, i1, lo2, hi2, ida)) continue;
     if (i1 - i0 + 1 > kTouchLong) {
       const int pos = atomicAdd(&qn, 1);
       if (pos < kTouchQ) {
@@ -149,7 +156,7 @@ __global__ void __launch_bounds__(256) k_touch(TouchP p) {
         continue;
       }
     }
-    for (int64_t i = i0; i <= i1; ++i) touch_slab(p, k, m, e, rows, i, lo2, hi2);
+    for (int64_t i = i0; i <= i1; ++i) touch_slab(p, k, m, e, rows, i, lo2, hi2, ida);
   }
   __syncthreads();
   const int nq = min(qn, kTouchQ);
@@ -158,8 +165,9 @@ __global__ void __launch_bounds__(256) k_touch(TouchP p) {
     const Edge e = p.edges[q[qi]];
     bool rows;
     int64_t i0, i1, lo2, hi2;
-    edge_slabs(p, e, rows, i0, i1, lo2, hi2);
-    for (int64_t i = i0 + lane; i <= i1; i += 32) touch_slab(p, k, m, e, rows, i, lo2, hi2);
+    double ida;
+    edge_slabs(p, e, rows, i0, i1, lo2, hi2, ida);
+    for (int64_t i = i0 + lane; i <= i1; i += 32) touch_slab(p, k, m, e, rows, i, lo2, hi2, ida);
   }
 }
 
@@ -178,6 +186,8 @@ cudaError_t launch_touch(Ctx& c, const int32_t* remap, cudaStream_t s) {
   p.remap = remap;
   p.pbits = c.d_pbits.as<uint32_t>();
   p.wpo = (c.rp.T + 31) / 32;
+  p.igt1 = 1.0 / c.geo.gt1;
+  p.igt5 = 1.0 / c.geo.gt5;
   k_touch<<<(unsigned)c.P, 256, 0, s>>>(p);
   c.launches += 1;
   return cudaGetLastError();
