@@ -409,7 +409,7 @@ def main():
                                parallelism=f"tile-row shards x{world}" + (" (shared GPU, gloo)" if shared else "")
                                + ("" if world == 1 else (" equal" if args.equal_shards else " work-balanced")),
                                l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA",
-                               cells="closed rectangle meets polygon (R15)" if args.cover else "centre inside"),
+                               semantics="closed rectangle meets polygon (R15)" if args.cover else "centre inside"),
                 "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
                 "clocks": clocks, "path": path, "steps_detail": steps_detail, "other_path": other,
                 "pairs": {k: st[k] for k in ("n_tiles", "n_candidates", "n_inside", "n_isect", "n_band_entries",

@@ -10,7 +10,9 @@ centres PAPER.md:18 §III.D, Franklin's ray-crossing test PAPER.md:20 Fig. 5) an
 reading taken where the paper is silent (also DESIGN.md §3).
 
 Parity status: pinned (tests/test_oracle_pins.py) — hand-worked counts, Fig. 5 crossing
-counts, closed-form histograms, np.bincount, the tiling partition invariant, O0 == O1.
+counts, closed-form histograms, np.bincount, the tiling partition invariant, O0 == O1.  The cover
+variant (reading R15) is pinned in tests/test_oracle_cover.py — closed forms and an exact
+rational-arithmetic reference on dyadic polygons.
 """
 from __future__ import annotations
 

@@ -23,7 +23,9 @@
  *   R8 canonical edge orientation: endpoints ordered so that ya <= yb before evaluating
  *      Franklin's expression xi = (xb - xa) * (yc - ya) / (yb - ya) + xa, left to right;
  *   R9 rings given by offsets, closed implicitly (edge v_{n-1} -> v_0);
- *   R10 half-open crossing rule: edge straddles iff ya <= yc < yb; crossing iff xc < xi.
+ *   R10 half-open crossing rule: edge straddles iff ya <= yc < yb; crossing iff xc < xi;
+ *   R15 (cover variant only) "geometrically intersect": closed cell rectangle meets the closed
+ *       polygon (see zho_cover_o0 at the end of this file).
  *
  * Functions:
  *   zho_bin            R3/R4 value -> bin (or -1)
