@@ -56,8 +56,10 @@ def _worker(rank, world, port, q):
         R = fill_host(cfg.dem, cfg.cols, r0, 0, r1 - r0, cfg.cols, nthreads=2)
         H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata), row0=r0, nthreads=2)
         t = torch.from_numpy(H.view(np.int64).copy())
-        reduce_histograms(t)
-        q.put((rank, t.numpy().view(np.uint64).copy()))
+        t0 = t.clone()
+        reduce_histograms(t)                  # all-reduce: every rank holds the sum
+        reduce_histograms(t0, to_rank0=True)  # reduce: rank 0 holds the sum (what bench.py uses)
+        q.put((rank, (t.numpy().view(np.uint64).copy(), t0.numpy().view(np.uint64).copy())))
     finally:
         dist.destroy_process_group()
 
@@ -81,4 +83,5 @@ def test_gloo_world2_reduce_equals_single_process():
     R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
     H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata))
     for r in range(world):
-        assert (res[r] == H).all()
+        assert (res[r][0] == H).all()
+    assert (res[0][1] == H).all()

@@ -46,7 +46,7 @@ def _worker(rank, world, port, cfg_name, q):
                                    row0=r0, nodata=cfg.nodata, fused=fused) as z:
                 z.set_output(out)
                 z.zh_run(None)
-            reduce_histograms(out)
+            reduce_histograms(out, to_rank0=fused)  # four-step: all-reduce; fused: reduce to rank 0 (bench.py)
             res.append(out.cpu().numpy().view(np.uint64).copy())
         q.put((rank, res[0], res[1]))
     finally:
@@ -86,9 +86,10 @@ def test_two_ranks_reduce_to_oracle(cuda_device, cfg_name):
             win = fill_host(cfg.dem, cfg.cols, r0, c0, r1 - r0, c1 - c0)
             want[k] = oracle.o1(win, cfg.gt, P.subset([k]), bins, row0=r0, col0=c0)[0]
     for rank, four, fused in got:
-        assert (four == fused).all()
         for k in rows:
-            assert (fused[k] == want[k]).all(), (rank, k)
+            assert (four[k] == want[k]).all(), (rank, k)
+            if rank == 0:
+                assert (fused[k] == want[k]).all(), (rank, k)
 
 
 def test_plan_rows_balanced_shards(cuda_device):
