@@ -63,14 +63,25 @@ def test_pip_predicate_has_no_contracted_fma():
     double division is an MUFU.RCP64H followed by a handful of DFMAs)."""
     from paper_conf_ipps_zhangw14_b200 import _build
     funcs = _sass_functions(_build.build())
-    names = [n for n in funcs if any(k in n for k in ("k_pipILi", "k_classify", "k_edges"))]
-    assert names
+    names = [n for n in funcs if any(k in n for k in ("k_pipILi", "k_parity", "k_classify", "k_edges"))]
+    assert any("k_parity" in n for n in names)
     for n in names:
         sass = "\n".join(funcs[n])
         assert "DMUL" in sass and "DADD" in sass, n
         n_rcp = sass.count("MUFU.RCP64H")
         assert n_rcp >= 1, n
         assert sass.count("DFMA") <= 10 * n_rcp, n
+
+
+def test_cover_segment_test_is_not_contracted():
+    """R15's segment-vs-cell test (k_touch) is written with __dsub_rn/__dmul_rn: its orientation
+    products must appear as DMUL, never fused into a DFMA with the following subtraction."""
+    from paper_conf_ipps_zhangw14_b200 import _build
+    funcs = _sass_functions(_build.build())
+    names = [n for n in funcs if "k_touch" in n]
+    assert names
+    sass = "\n".join(funcs[names[0]])
+    assert sass.count("DMUL") >= 8  # two products per corner, four corners
 
 
 def _mk(lib_zh, **over):

@@ -20,4 +20,9 @@ for tile, fused in ((128, False), (128, True), (100, True), (100, False)):
         res.append(z.run())
         z.zh_zonal_stats()
 assert all((r == res[0]).all() for r in res)
+cov = []
+for tile, fused in ((128, True), (100, False)):  # cover mode (R15): k_touch on top of the split step 4
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=tile, nodata=cfg.nodata, fused=fused, cover=True) as z:
+        cov.append(z.run())
+assert (cov[0] == cov[1]).all() and (cov[0] >= res[0]).all()
 print("sanitize run ok", int(res[0].sum()))
