@@ -17,6 +17,10 @@
 #include "zh_pip.cuh"
 #include "zh_tilehist.cuh"
 
+#ifndef ZH_EXACT_GRID
+#define ZH_EXACT_GRID 1  // 1: step-4 grids sized from the list counts (host reads them during k_fused_pure)
+#endif
+
 #ifndef ZH_PAR_SIDE
 #define ZH_PAR_SIDE 0  // 1: k_parity on the side stream, beside k_fused_pure (measured slower: registers)
 #endif
@@ -93,7 +97,7 @@ __global__ void k_pure_tiles(const uint32_t* __restrict__ pure_cnt, int64_t n, c
 // tile run back to back and all but the first find its cells in L2 (grouped by polygon, as step 2
 // emits them, the L2 hit rate of k_pip was 15 %).
 __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, const int2* __restrict__ inside,
-                           int64_t n_inside, const uint32_t* __restrict__ extra, const uint32_t* __restrict__ pip_off,
+                           int64_t n_inside, const uint32_t* __restrict__ extra, const uint64_t* __restrict__ pip_off,
                            uint32_t* __restrict__ cursor, int64_t n_tiles, RasterP rp, int2* __restrict__ pip,
                            int32_t* __restrict__ remap, int64_t* __restrict__ counts) {
   const int64_t n = n_isect + n_inside;
@@ -106,15 +110,37 @@ __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, cons
       if (!extra[i - n_isect]) continue;
       pr = inside[i - n_isect];
     }
-    const uint32_t pos = pip_off[pr.x] + atomicAdd(&cursor[pr.x], 1u);
+    const uint32_t pos = (uint32_t)pip_off[pr.x] + atomicAdd(&cursor[pr.x], 1u);
     pip[pos] = pr;
     if (remap && i < n_isect) remap[i] = (int32_t)pos;  // isect index -> list index (k_touch)
     cells += tile_cells(rp, pr.x);
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) counts[1] = (int64_t)pip_off[n_tiles];
+  if (blockIdx.x == 0 && threadIdx.x == 0) counts[1] = (int64_t)(uint32_t)pip_off[n_tiles];
   for (int o = 16; o > 0; o >>= 1) cells += __shfl_xor_sync(0xffffffffu, cells, o);
   if ((threadIdx.x & 31) == 0 && cells) atomicAdd(reinterpret_cast<unsigned long long*>(&counts[3]),
                                                   (unsigned long long)cells);
+}
+
+// Tile groups of the grouped cell kernel (k_mixed_cells): a mixed tile with c cell-in-polygon pairs
+// forms ceil(c / 2) groups of <= 2 consecutive pairs.  pk[t] = c | ceil(c / 2) << 32, so one
+// exclusive scan gives both the tile's first pair (low half) and its first group (high half).
+__global__ void k_pack_mixed(const uint32_t* __restrict__ cnt, int64_t n, uint64_t* __restrict__ pk) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = cnt[i];
+    pk[i] = (uint64_t)c | ((uint64_t)((c + 1) >> 1) << 32);
+  }
+}
+
+// grp[g] = {first pair index, #pairs}; counts[4] = #groups
+__global__ void k_pip_groups(const uint32_t* __restrict__ cnt, const uint64_t* __restrict__ off, int64_t n_tiles,
+                             int2* __restrict__ grp, int64_t* __restrict__ counts) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n_tiles; t += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = cnt[t];
+    if (!c) continue;
+    const uint32_t p0 = (uint32_t)off[t], g0 = (uint32_t)(off[t] >> 32);
+    for (uint32_t q = 0; 2 * q < c; ++q) grp[g0 + q] = make_int2((int)(p0 + 2 * q), (int)min(2u, c - 2 * q));
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) counts[4] = (int64_t)(off[n_tiles] >> 32);
 }
 
 struct PureP {
@@ -248,11 +274,12 @@ cudaError_t launch_fused(Ctx& c) {
   if ((e = c.d_pure_poly.ensure(sizeof(int32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
   if ((e = c.d_pure_tiles.ensure(sizeof(int32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
   if ((e = c.d_extra.ensure(sizeof(uint32_t) * ((size_t)NI + 1))) != cudaSuccess) return e;
-  if ((e = c.d_extra_pos.ensure(sizeof(uint32_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_extra_pos.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
+  if ((e = c.d_mixed_pk.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pip.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
-  if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 4)) != cudaSuccess) return e;
+  if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 6)) != cudaSuccess) return e;
   if (c.cover && (e = c.d_remap.ensure(sizeof(int32_t) * ((size_t)NX + 1))) != cudaSuccess) return e;
-  cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 4, c.stream);
+  cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 6, c.stream);
   if (NT == 0 || NI + NX == 0) {
     if (c.timing)
       for (int i = 10; i < 16; ++i) cudaEventRecord(c.ev[i], c.stream);
@@ -286,14 +313,26 @@ cudaError_t launch_fused(Ctx& c) {
   k_pure_tiles<<<grid_for(NT, 256), 256, 0, c.stream>>>(c.d_pure_cnt.as<uint32_t>(), NT, c.d_pure_off.as<uint64_t>(),
                                                         c.rp, c.d_pure_tiles.as<int32_t>(), c.d_fcounts.as<int64_t>());
   c.launches += 1;
-  if ((e = excl_scan<uint32_t>(c, c.d_mixed.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(), NT + 1)) != cudaSuccess)
+  k_pack_mixed<<<grid_for(NT + 1, 256), 256, 0, c.stream>>>(c.d_mixed.as<uint32_t>(), NT + 1,
+                                                            c.d_mixed_pk.as<uint64_t>());
+  c.launches += 1;
+  if ((e = excl_scan<uint64_t>(c, c.d_mixed_pk.as<uint64_t>(), c.d_extra_pos.as<uint64_t>(), NT + 1)) != cudaSuccess)
     return e;
   k_pip_list<<<grid_for(NI + NX, 256), 256, 0, c.stream>>>(c.d_isect.as<int2>(), NX, c.d_inside.as<int2>(), NI,
-                                                          c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint32_t>(),
+                                                          c.d_extra.as<uint32_t>(), c.d_extra_pos.as<uint64_t>(),
                                                           c.d_pip_cur.as<uint32_t>(), NT, c.rp, c.d_pip.as<int2>(),
                                                           c.cover ? c.d_remap.as<int32_t>() : nullptr,
                                                           c.d_fcounts.as<int64_t>());
   c.launches += 1;
+
+  // grouped cell kernel: tile groups of <= 2 pairs (every cell read once per group)
+  const bool grouped = c.pip_group != 0 && mixed_smem(c) > 0;
+  if (grouped) {
+    if ((e = c.d_pip_grp.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
+    k_pip_groups<<<grid_for(NT, 256), 256, 0, c.stream>>>(c.d_mixed.as<uint32_t>(), c.d_extra_pos.as<uint64_t>(), NT,
+                                                          c.d_pip_grp.as<int2>(), c.d_fcounts.as<int64_t>());
+    c.launches += 1;
+  }
 
   const int mode = fast_bins_ok(c.bp) ? (make_fast_bins(c.bp).bias ? 4 : (c.bp.use_nodata ? 3 : 2))
                                       : (c.bp.width == 1 ? 0 : 1);
@@ -301,18 +340,33 @@ cudaError_t launch_fused(Ctx& c) {
   // stream WHILE the pure-tile kernel streams the pure tiles (FP64-latency work beside HBM-bound
   // work), then the cell kernel runs once both are done
   const bool split = c.pip_split != 0 || c.cover != 0;
+  // exact grids for the step-4 kernels: the list sizes are copied to the host behind the list
+  // kernels and read while the pure-tile kernel runs (no CTAs that only find they have no work)
+  const bool exact = split && ZH_EXACT_GRID;
+  int64_t n_pip = NI + NX, n_grp = NI + NX;
   if (split) {
     if ((e = pip_prepare(c, NI + NX)) != cudaSuccess) return e;
-    cudaEventRecord(c.ev_fork, c.stream);
-    cudaStreamWaitEvent(c.side, c.ev_fork, 0);
+  }
+  if (exact) {
+    cudaMemcpyAsync(c.pinned_counts + 8, c.d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c.stream);
+    cudaEventRecord(c.ev_counts, c.stream);
+  }
+  auto parity = [&](int64_t grid) -> cudaError_t {
+    cudaError_t pe;
     if (c.timing) cudaEventRecord(c.ev[13], ZH_PAR_SIDE ? c.side : c.stream);
-    if ((e = launch_parity(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1,
-                           ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess)
-      return e;
+    if ((pe = launch_parity(c, c.d_pip.as<int2>(), grid, c.d_fcounts.as<int64_t>() + 1,
+                            ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess)
+      return pe;
     if (c.cover) {  // R15: cells an edge reaches join the parity bits (k_touch.cu)
-      if ((e = launch_touch(c, c.d_remap.as<int32_t>(), ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess) return e;
+      if ((pe = launch_touch(c, c.d_remap.as<int32_t>(), ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess) return pe;
     }
     if (c.timing) cudaEventRecord(c.ev[14], ZH_PAR_SIDE ? c.side : c.stream);
+    return cudaSuccess;
+  };
+  if (split && !exact) {
+    cudaEventRecord(c.ev_fork, c.stream);
+    cudaStreamWaitEvent(c.side, c.ev_fork, 0);
+    if ((e = parity(NI + NX)) != cudaSuccess) return e;
     cudaEventRecord(c.ev_join, c.side);
   }
   // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
@@ -342,9 +396,26 @@ cudaError_t launch_fused(Ctx& c) {
   }
   if (c.timing) cudaEventRecord(c.ev[11], c.stream);
   if (split) {
-    cudaStreamWaitEvent(c.stream, c.ev_join, 0);
+    if (exact) {
+      if ((e = cudaEventSynchronize(c.ev_counts)) != cudaSuccess) return e;
+      n_pip = c.pinned_counts[8 + 1];
+      n_grp = c.pinned_counts[8 + 4];
+      if (n_pip > 0) {
+        if ((e = parity(n_pip)) != cudaSuccess) return e;
+      } else if (c.timing) {
+        cudaEventRecord(c.ev[13], c.stream);
+        cudaEventRecord(c.ev[14], c.stream);
+      }
+    } else {
+      cudaStreamWaitEvent(c.stream, c.ev_join, 0);
+    }
     if (c.timing) cudaEventRecord(c.ev[15], c.stream);
-    e = launch_pip_cells(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1);
+    if (grouped)
+      e = n_grp > 0 ? launch_mixed_cells(c, c.d_pip.as<int2>(), c.d_pip_grp.as<int2>(), n_grp,
+                                         c.d_fcounts.as<int64_t>() + 4)
+                    : cudaSuccess;
+    else
+      e = n_pip > 0 ? launch_pip_cells(c, c.d_pip.as<int2>(), n_pip, c.d_fcounts.as<int64_t>() + 1) : cudaSuccess;
   } else {
     if (c.timing) {
       cudaEventRecord(c.ev[13], c.stream);

@@ -21,6 +21,8 @@
 //     one branch-free shared atomic per cell; vectors with no inside cell are not even loaded)
 //     into a CTA-private shared histogram, flushed once per pair with one global atomic per
 //     non-zero bin (no race).
+#include <algorithm>
+
 #include "zh_ctx.h"
 #include "zh_pip.cuh"
 
@@ -64,6 +66,20 @@ __global__ void __launch_bounds__(kPipThreads, ZH_PIP_MINB) k_pip_cells(PipP p) 
   pip_cells_body<kMode, kU64>(p, blockIdx.x, sh);
 }
 
+#ifndef ZH_MIX_THREADS
+#define ZH_MIX_THREADS 256
+#endif
+#ifndef ZH_MIX_MINB
+#define ZH_MIX_MINB 4
+#endif
+// Tile groups of <= 2 pairs (fused path): each cell read once per group (zh_pip.cuh).
+template <int kMode, bool kU64>
+__global__ void __launch_bounds__(ZH_MIX_THREADS, ZH_MIX_MINB) k_mixed_cells(PipP p) {
+  if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
+  extern __shared__ __align__(16) uint32_t sh[];
+  mixed_cells_body<kMode, kU64>(p, blockIdx.x, sh);
+}
+
 cudaError_t launch_pip(Ctx& c) { return launch_pip_list(c, c.d_isect.as<int2>(), c.n_isect, nullptr); }
 
 
@@ -96,6 +112,7 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev) {
   if (p.rcc < 1) p.rcc = 1;
   if (p.rcc > c.rp.T) p.rcc = c.rp.T;
   p.pbits = c.d_pbits.as<uint32_t>();
+  p.grp = nullptr;
   return p;
 }
 
@@ -141,6 +158,43 @@ cudaError_t launch_pip_cells(Ctx& c, const int2* pairs, int64_t grid, const int6
   }
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k<<<(unsigned)grid, kPipThreads, smem, c.stream>>>(p);
+  c.launches += 1;
+  return cudaGetLastError();
+}
+
+// Rows per staged bitmap chunk of k_mixed_cells: 4 KB per pair (4 CTAs of 48 KB per SM at 5,000 bins).
+static int mixed_rows(const Ctx& c) {
+  const int wpo = (c.rp.T + 31) / 32;
+  return std::max(1, std::min(c.rp.T, 1024 / wpo));
+}
+
+// Shared memory of k_mixed_cells, or 0 when the grouped form does not apply (two histograms must
+// fit the CTA, and the packed form needs 16-bit byte offsets over both).
+
+size_t mixed_smem(Ctx& c) {
+  const size_t hw = (size_t)hist_words(c.bp.nbins);
+  const size_t smem = 2 * hw * 4 + 2 * (size_t)mixed_rows(c) * ((c.rp.T + 31) / 32) * 4;
+  if (smem > 200 * 1024) return 0;
+  if (pip_mode(c) >= 2 && 2 * hw * 4 >= 65536) return 0;
+  return smem;
+}
+
+cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64_t grid, const int64_t* n_dev) {
+  if (grid == 0) return cudaSuccess;
+  PipP p = pip_params(c, pairs, n_dev);
+  p.grp = grp;
+  p.rcc = mixed_rows(c);
+  const size_t smem = mixed_smem(c);
+  void (*k)(PipP);
+  switch (pip_mode(c)) {
+    case 0: k = c.out_u64 ? k_mixed_cells<0, true> : k_mixed_cells<0, false>; break;
+    case 1: k = c.out_u64 ? k_mixed_cells<1, true> : k_mixed_cells<1, false>; break;
+    case 2: k = c.out_u64 ? k_mixed_cells<2, true> : k_mixed_cells<2, false>; break;
+    case 3: k = c.out_u64 ? k_mixed_cells<3, true> : k_mixed_cells<3, false>; break;
+    default: k = c.out_u64 ? k_mixed_cells<4, true> : k_mixed_cells<4, false>; break;
+  }
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k<<<(unsigned)grid, ZH_MIX_THREADS, smem, c.stream>>>(p);
   c.launches += 1;
   return cudaGetLastError();
 }

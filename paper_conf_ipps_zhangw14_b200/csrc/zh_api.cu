@@ -190,13 +190,14 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
     c->rp.data = c->raster_dev.as<int16_t>();
     if (r->pitch % 8 != 0) return cleanup_fail(fail(ZH_ERR_INVALID_ARG, "host raster pitch must be a multiple of 8"));
   }
-  if ((e = cudaHostAlloc((void**)&c->pinned_counts, 8 * sizeof(int64_t), cudaHostAllocDefault)) != cudaSuccess)
+  if ((e = cudaHostAlloc((void**)&c->pinned_counts, 16 * sizeof(int64_t), cudaHostAllocDefault)) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (pinned counters)"));
   for (int i = 0; i < 16; ++i)
     if ((e = cudaEventCreate(&c->ev[i])) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (events)"));
   if ((e = cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming)) != cudaSuccess ||
-      (e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming)) != cudaSuccess)
+      (e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_counts, cudaEventDisableTiming)) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (side stream)"));
   if ((e = cudaGetLastError()) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
   *out = reinterpret_cast<zh_ctx>(c);
@@ -213,7 +214,8 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_class, &c->d_flags, &c->d_flag_pos, &c->d_inside, &c->d_isect, &c->d_counts,
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
-                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats};
+                      &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats,
+                      &c->d_pip_grp, &c->d_mixed_pk};
   for (auto* b : bufs) b->release();
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
@@ -223,6 +225,7 @@ extern "C" void zh_destroy(zh_ctx h) {
   }
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
+  if (c->ev_counts) cudaEventDestroy(c->ev_counts);
   if (c->pinned_counts) cudaFreeHost(c->pinned_counts);
   delete c;
 }
@@ -234,7 +237,8 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_class, &c.d_flags, &c.d_flag_pos, &c.d_inside, &c.d_isect, &c.d_counts,
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
-                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats};
+                            &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats,
+                            &c.d_pip_grp, &c.d_mixed_pk};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;

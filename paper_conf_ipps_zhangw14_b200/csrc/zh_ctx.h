@@ -7,6 +7,9 @@
 
 #include "zh_internal.cuh"
 
+#ifndef ZH_PIP_GROUP_DEFAULT
+#define ZH_PIP_GROUP_DEFAULT 1
+#endif
 #ifndef ZH_PIP_SPLIT_DEFAULT
 #define ZH_PIP_SPLIT_DEFAULT 1
 #endif
@@ -49,6 +52,7 @@ struct Ctx {
   int32_t out_u64 = 1;
   int32_t force_isect = 0;
   int32_t cover = 0;  // R15: closed cell rectangle meets the closed polygon (k_touch.cu)
+  int32_t pip_group = ZH_PIP_GROUP_DEFAULT;  // fused path: mixed-tile groups of <= 2 pairs (k_mixed_cells) or one CTA per pair
   int32_t pip_split = ZH_PIP_SPLIT_DEFAULT;  // step 4 as k_parity + k_pip_cells (1) or one k_pip kernel per pair (0)
   cudaStream_t stream = nullptr;
   // polygons (device)
@@ -60,7 +64,7 @@ struct Ctx {
   DBuf d_inside, d_isect, d_counts, d_cub;
   // fused path lists (k_fused.cu)
   DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,
-      d_pip, d_pip_cur, d_fcounts, d_pbits, d_remap;
+      d_pip, d_pip_cur, d_fcounts, d_pbits, d_remap, d_pip_grp, d_mixed_pk;
   DBuf d_stats;  // zonal statistics [P][8] (k_stats.cu)
   int64_t n_cand = 0, n_bands = 0, n_band_entries = 0, n_inside = 0, n_isect = 0;
   // step 1 product and output
@@ -76,6 +80,7 @@ struct Ctx {
   cudaEvent_t ev[16] = {};  // start/stop per timed call: steps 1..4, fused; + fused inner marks 10..15
   cudaStream_t side = nullptr;            // second stream of the fused path (k_parity beside k_fused_pure)
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  cudaEvent_t ev_counts = nullptr;        // fused path: list sizes copied to pinned_counts[8..13]
   int64_t fused_counts[4] = {0, 0, 0, 0};  // pure tiles, pip pairs, pure cells, pip cells
   int64_t launches = 0;
   int64_t host_count_buf[4] = {0, 0, 0, 0};
@@ -92,6 +97,8 @@ cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64
 cudaError_t pip_prepare(Ctx& c, int64_t grid);  // split form: per-pair parity bitmap buffer
 cudaError_t launch_parity(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev, cudaStream_t s);
 cudaError_t launch_pip_cells(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
+size_t mixed_smem(Ctx& c);  // 0: the grouped cell kernel does not apply
+cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64_t grid, const int64_t* n_dev);
 cudaError_t launch_touch(Ctx& c, const int32_t* remap, cudaStream_t s);  // k_touch.cu (cover mode)
 cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
 cudaError_t launch_zonal_stats(Ctx& c, int64_t* dstats);  // k_stats.cu

@@ -210,6 +210,29 @@ __device__ __forceinline__ void count8_fast(uint32_t* __restrict__ hist, const u
   }
 }
 
+// Two histograms side by side (words [0, hw) and [hw, 2 hw)): as count8_fast, and cell j goes to
+// the second one when bit j of `sel` is set.  `off2` = hw in both halves; the slot offset is added
+// after the dummy clamp, so a selected cell that is not counted lands on the second histogram's
+// dummy slot (never flushed).  Byte offsets stay 16-bit: the caller guarantees 2 hw * 4 < 2^16.
+template <int kForm>
+__device__ __forceinline__ void count8_fast_sel(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                                uint32_t sel, const FastBins& f, uint32_t dum2, uint32_t off2) {
+  uint32_t sl, sh, el, eh;
+  spread_bits8(skip, sl, sh);
+  spread_bits8(sel, el, eh);
+  const uint32_t ws[4] = {q.x, q.y, q.z, q.w};
+  char* hb = reinterpret_cast<char*>(hist);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t P = (uint32_t)((2 * i) | (2 * i) << 4 | (2 * i + 1) << 8 | (2 * i + 1) << 12);
+    uint32_t x = fast_idx2<kForm>(ws[i], f) | __byte_perm(sl, sh, P);
+    x = __vminu2(x, dum2);
+    x = (x + (__byte_perm(el, eh, P) & off2)) << 2;  // halves < 2 hw: no carry between them
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);
+  }
+}
+
 // Generic path (any width / lo / nbins): same layout, scalar mapping, per-cell atomics.
 template <bool kW1>
 __device__ __forceinline__ void count8_generic(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
@@ -218,6 +241,17 @@ __device__ __forceinline__ void count8_generic(uint32_t* __restrict__ hist, cons
   for (int j = 0; j < 8; ++j) {
     int b = ((skip >> j) & 1u) ? -1 : bin_of<kW1>(cell_of(q, j), bp);
     atomicAdd(&hist[b >= 0 ? kOff + b : (int)dummy], 1u);
+  }
+}
+
+// Generic path of count8_fast_sel: cell j goes to hist + hw when bit j of `sel` is set.
+template <bool kW1>
+__device__ __forceinline__ void count8_generic_sel(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                                   uint32_t sel, const BinP& bp, uint32_t dummy, int hw) {
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    int b = ((skip >> j) & 1u) ? -1 : bin_of<kW1>(cell_of(q, j), bp);
+    atomicAdd(&hist[(b >= 0 ? kOff + b : (int)dummy) + (((sel >> j) & 1u) ? hw : 0)], 1u);
   }
 }
 

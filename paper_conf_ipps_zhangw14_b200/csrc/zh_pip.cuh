@@ -4,6 +4,10 @@
 
 #include "zh_parity.cuh"
 
+#ifndef ZH_MIX_ROWS4
+#define ZH_MIX_ROWS4 1
+#endif
+
 namespace zh {
 
 struct PipP {
@@ -26,6 +30,7 @@ struct PipP {
   uint32_t* pbits;       // split form: per-pair parity bitmaps [pair][T][wpo] (global)
   int wpo;               // words per stored parity row = ceil(T / 32)
   int rcc;               // rows per chunk of the split cell kernel's shared copy of the bitmap
+  const int2* grp;       // tile groups of the cell kernel: {first pair index, #pairs (1 or 2)}
 };
 
 struct Ctx;  // zh_ctx.h
@@ -292,6 +297,186 @@ __device__ __forceinline__ void pip_cells_body(const PipP& p, int64_t pair_idx, 
       }
     }
   }
+}
+
+// Add the shared histogram `hist` (HistLayout) into output row k (one global atomic per non-zero bin).
+template <bool kU64>
+__device__ __forceinline__ void flush_hist(const uint32_t* __restrict__ hist, int nbins, int k, void* out) {
+  const int64_t orow = (int64_t)k * nbins;
+  for (int b = threadIdx.x * 4; b < nbins; b += blockDim.x * 4) {  // 16-byte reads, zero vectors skipped
+    const uint4 v = *reinterpret_cast<const uint4*>(&hist[kOff + b]);
+    if (!(v.x | v.y | v.z | v.w)) continue;
+    const uint32_t vs[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (vs[q] && b + q < nbins) {
+        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(out) + orow + b + q, (unsigned long long)vs[q]);
+        else atomicAdd(reinterpret_cast<uint32_t*>(out) + orow + b + q, vs[q]);
+      }
+    }
+  }
+}
+
+// Cells of a GROUP of pairs of one mixed tile (p.grp[g] = {first pair index, m}, m = 1 or 2; the
+// pair list is grouped by tile), with the parity bitmaps of k_parity: each 16-byte vector is read
+// ONCE for both pairs.  When no cell of the tile is inside both polygons (always, for polygons that
+// partition the plane), each cell goes to exactly one of two shared histograms (count8_fast_sel:
+// one atomic per cell, whatever m).  Otherwise (overlapping polygons, cover mode) every vector is
+// counted once per pair.  The branch is uniform over the CTA (__syncthreads_or of the overlap).
+// `sh` holds 2 hist_words(nbins) + 2 rcc * wpo words.
+template <int kMode, bool kU64>
+__device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint32_t* __restrict__ sh) {
+  const int HW = hist_words(p.bp.nbins);
+  const int2 gr = p.grp[g];
+  const int64_t pi0 = gr.x;
+  const int m = gr.y;
+  uint32_t* hist = sh;
+  uint32_t* bm0 = sh + 2 * HW;
+  uint32_t* bm1 = bm0 + p.rcc * p.wpo;
+  const RasterP& rp = p.rp;
+  const int2 pr0 = p.isect[pi0];
+  const int tile = pr0.x;
+  const int kp0 = pr0.y, kp1 = m > 1 ? p.isect[pi0 + 1].y : -1;
+  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int64_t r0 = (int64_t)(rp.tr0 + trl) * rp.T, c0 = (int64_t)tc * rp.T;
+  const int h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - r0);
+  const int w = (int)min((int64_t)rp.T, rp.cols - c0);
+  const int wpo = p.wpo;
+  const uint32_t* __restrict__ src0 = p.pbits + pi0 * (int64_t)rp.T * wpo;
+  const uint32_t* __restrict__ src1 = src0 + (int64_t)rp.T * wpo;
+
+  for (int i = threadIdx.x * 4; i < m * HW; i += blockDim.x * 4)
+    *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
+  const uint32_t dummy = (uint32_t)hist_dummy(p.bp.nbins) + (threadIdx.x & 31);
+  const uint32_t dum2 = dummy * 0x10001u;
+  const uint32_t off2 = (uint32_t)HW * 0x10001u;
+  const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
+  const int nk = (int)(k1 - k0);
+  const int64_t pitch = rp.pitch;
+  const FastBins fb = p.fb;
+  auto count = [&](const uint4& q, uint32_t skip, uint32_t* hh) {
+    if (kMode >= 2) count8_fast<kMode - 2, true>(hh, q, skip, fb, dum2);
+    else count8_generic<kMode == 0>(hh, q, skip, p.bp, dummy);
+  };
+  auto count_sel = [&](const uint4& q, uint32_t skip, uint32_t sel) {
+    if (kMode >= 2) count8_fast_sel<kMode - 2>(hist, q, skip, sel, fb, dum2, off2);
+    else count8_generic_sel<kMode == 0>(hist, q, skip, sel, p.bp, dummy, HW);
+  };
+
+  for (int cr = 0; cr < h; cr += p.rcc) {
+    const int ch = min(p.rcc, h - cr);
+    uint32_t ov = 0;
+    if ((wpo & 3) == 0) {
+      const uint4* s0 = reinterpret_cast<const uint4*>(src0 + (int64_t)cr * wpo);
+      const uint4* s1 = reinterpret_cast<const uint4*>(src1 + (int64_t)cr * wpo);
+      for (int i = threadIdx.x; i < ch * wpo / 4; i += blockDim.x) {
+        const uint4 a = __ldcs(s0 + i);
+        const uint4 b = m > 1 ? __ldcs(s1 + i) : make_uint4(0, 0, 0, 0);
+        reinterpret_cast<uint4*>(bm0)[i] = a;
+        reinterpret_cast<uint4*>(bm1)[i] = b;
+        ov |= (a.x & b.x) | (a.y & b.y) | (a.z & b.z) | (a.w & b.w);
+      }
+    } else {
+      const uint32_t* s0 = src0 + (int64_t)cr * wpo;
+      const uint32_t* s1 = src1 + (int64_t)cr * wpo;
+      for (int i = threadIdx.x; i < ch * wpo; i += blockDim.x) {
+        const uint32_t a = __ldcs(s0 + i), b = m > 1 ? __ldcs(s1 + i) : 0u;
+        bm0[i] = a;
+        bm1[i] = b;
+        ov |= a & b;
+      }
+    }
+    const bool overlap = __syncthreads_or(ov != 0) != 0;
+    const int16_t* base = rp.data + (r0 + cr - rp.row0) * pitch + k0 * 8;
+    if (nk <= (int)blockDim.x) {
+      const int rpi = blockDim.x / nk;
+      const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
+      auto run = [&](auto aligned, auto ovl) {
+        constexpr bool kA = decltype(aligned)::value;
+        constexpr bool kO = decltype(ovl)::value;
+        const int64_t cs = (k0 + kk) * 8;
+        const uint32_t cskip = cols_skip8(cs, c0, w);
+        const int lc0 = (int)(cs - c0);
+        const int wi = lc0 >> 5, bsh = lc0 & 31;
+        auto pbits = [&](const uint32_t* bm, int lr) -> uint32_t {
+          if (kA) return (bm[lr * wpo + wi] >> bsh) & 0xFFu;
+          return bits8(bm + lr * wpo, wpo, lc0);
+        };
+        const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
+        const int64_t step = (int64_t)rpi * pitch;
+        int lr = rs;
+        if (!kO) {
+#if ZH_MIX_ROWS4
+          // four rows per iteration: four 16-byte loads in flight per thread
+          for (; lr + 3 * rpi < ch; lr += 4 * rpi, ptr += 4 * step) {
+            uint32_t e[4], s[4];
+            uint4 q[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              e[u] = pbits(bm1, lr + u * rpi);
+              s[u] = cskip | (~(pbits(bm0, lr + u * rpi) | e[u]) & 0xFFu);
+              q[u] = make_uint4(0, 0, 0, 0);
+              if (s[u] != 0xFFu) q[u] = ld_stream16(ptr + u * step);
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              if (s[u] != 0xFFu) count_sel(q[u], s[u], e[u]);
+          }
+#endif
+          for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
+            const uint32_t e0 = pbits(bm1, lr), e1 = pbits(bm1, lr + rpi);
+            const uint32_t s0 = cskip | (~(pbits(bm0, lr) | e0) & 0xFFu);
+            const uint32_t s1 = cskip | (~(pbits(bm0, lr + rpi) | e1) & 0xFFu);
+            uint4 q0 = make_uint4(0, 0, 0, 0), q1 = make_uint4(0, 0, 0, 0);
+            if (s0 != 0xFFu) q0 = ld_stream16(ptr);
+            if (s1 != 0xFFu) q1 = ld_stream16(ptr + step);
+            if (s0 != 0xFFu) count_sel(q0, s0, e0);
+            if (s1 != 0xFFu) count_sel(q1, s1, e1);
+          }
+          for (; lr < ch; lr += rpi, ptr += step) {
+            const uint32_t e = pbits(bm1, lr);
+            const uint32_t skip = cskip | (~(pbits(bm0, lr) | e) & 0xFFu);
+            if (skip == 0xFFu) continue;
+            count_sel(ld_stream16(ptr), skip, e);
+          }
+        } else {
+          for (; lr < ch; lr += rpi, ptr += step) {
+            const uint32_t s0 = cskip | (~pbits(bm0, lr) & 0xFFu);
+            const uint32_t s1 = cskip | (~pbits(bm1, lr) & 0xFFu);
+            if ((s0 & s1) == 0xFFu) continue;
+            const uint4 q = ld_stream16(ptr);
+            if (s0 != 0xFFu) count(q, s0, hist);
+            if (s1 != 0xFFu) count(q, s1, hist + HW);
+          }
+        }
+      };
+      if (rs < rpi) {
+        using T_ = std::integral_constant<bool, true>;
+        using F_ = std::integral_constant<bool, false>;
+        if ((c0 & 7) == 0) {
+          if (overlap) run(T_{}, T_{}); else run(T_{}, F_{});
+        } else {
+          if (overlap) run(F_{}, T_{}); else run(F_{}, F_{});
+        }
+      }
+    } else {
+      for (int lr = 0; lr < ch; ++lr) {
+        for (int kk = threadIdx.x; kk < nk; kk += blockDim.x) {
+          const int64_t cs = (k0 + kk) * 8;
+          const uint32_t cskip = cols_skip8(cs, c0, w);
+          const uint32_t s0 = cskip | (~bits8(bm0 + lr * wpo, wpo, (int)(cs - c0)) & 0xFFu);
+          const uint32_t s1 = cskip | (~bits8(bm1 + lr * wpo, wpo, (int)(cs - c0)) & 0xFFu);
+          if ((s0 & s1) == 0xFFu) continue;
+          const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
+          if (s0 != 0xFFu) count(q, s0, hist);
+          if (s1 != 0xFFu) count(q, s1, hist + HW);
+        }
+      }
+    }
+    __syncthreads();
+  }
+  flush_hist<kU64>(hist, p.bp.nbins, kp0, p.out);
+  if (m > 1) flush_hist<kU64>(hist + HW, p.bp.nbins, kp1, p.out);
 }
 
 }  // namespace zh
