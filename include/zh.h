@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 4
+#define ZH_ABI_VERSION 5
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -64,7 +64,9 @@ typedef enum {
  * on_host = 0: `data` is DEVICE memory (borrowed).  The fast paths need data % 16 == 0 and
  *   pitch % 8 == 0 (16-byte vector loads); other alignments are rejected (INVALID_ARG).
  * on_host = 1: `data` is HOST memory (borrowed; pin it for full PCIe speed); the context owns a
- *   device copy and every zh_run / zh_upload_raster copies the shard host->device first.
+ *   device copy.  zh_upload_raster copies the whole shard host->device; zh_run does too, except
+ *   with options.fused = 1, where it runs step 2 first and copies only the tiles that some
+ *   (tile, polygon) pair needs (the fused kernels never read the others; zh_stats.h2d_bytes).
  * Geotransform (GDAL): x = gt[0] + col*gt[1] + row*gt[2], y = gt[3] + col*gt[4] + row*gt[5];
  *   the cell (r, c) has centre x = gt[0] + (c + 0.5)*gt[1], y = gt[3] + (r + 0.5)*gt[5]
  *   (with options.rep_custom: (c + rep_x), (r + rep_y) instead of the 0.5s).
@@ -142,6 +144,8 @@ typedef struct {
   int64_t n_pip_pairs;    /* after zh_fused_update: pairs sent to the cell-in-polygon kernel      */
   int64_t n_pure_cells;   /* cells of those pure tiles                                          */
   int64_t n_pip_cells;    /* cells of the tiles of those pairs (counted once per pair)           */
+  int64_t h2d_bytes;      /* on_host rasters: bytes copied host->device by the last zh_run /
+                             zh_upload_raster                                                   */
 } zh_stats;
 
 /* Validate, copy polygons to the device (H2D on options->stream), allocate per-tile histograms
@@ -173,8 +177,18 @@ zh_status zh_pip_update(zh_ctx ctx);
 zh_status zh_fused_update(zh_ctx ctx);
 
 /* Upload (on_host), steps 2, 1, 3, 4 (or 2 + fused when options.fused), then copy n_poly * nbins elements (uint64 or uint32 per
- * out_u64, row-major [n_poly][nbins]) to host_out (may be NULL to skip the copy).  Syncs. */
+ * out_u64, row-major [n_poly][nbins]) to host_out (may be NULL to skip the copy).  Syncs.
+ * on_host with options.fused: the upload follows step 2 and covers only the needed tiles (see
+ * zh_raster). */
 zh_status zh_run(zh_ctx ctx, void* host_out);
+
+/* Device memory of destroyed contexts is kept in a process-wide cache and reused by later
+ * contexts of the same device (no cudaMalloc / cudaFree of the raster copy per zh_create /
+ * zh_destroy cycle); allocations that fail return the cache to the driver and retry.
+ * zh_trim_cache frees every cached block; keep_caching = 0 also disables caching from then on.
+ * zh_cache_bytes: bytes currently cached. */
+void zh_trim_cache(int32_t keep_caching);
+int64_t zh_cache_bytes(void);
 
 /* Zonal statistics from the histograms (the classic per-zone min, max, average,
  * count and standard deviation of PAPER.md:10 §I ¶1), exact integers in units of bin indices b

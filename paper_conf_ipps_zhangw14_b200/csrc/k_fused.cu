@@ -223,6 +223,15 @@ cudaError_t launch_row_cost(Ctx& c, double* d_row_cost) {
   return cudaGetLastError();
 }
 
+// need[t] = 1 for every tile of some inside or intersecting pair (on_host zh_run of the fused path
+// uploads only those tiles: the others are read by no kernel)
+__global__ void k_need_tiles(const int2* __restrict__ inside, int64_t n_inside, const int2* __restrict__ isect,
+                             int64_t n_isect, uint8_t* __restrict__ need) {
+  const int64_t n = n_inside + n_isect;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    need[i < n_inside ? inside[i].x : isect[i - n_inside].x] = 1;
+}
+
 static int grid_for(int64_t n, int threads) {
   int64_t b = (n + threads - 1) / threads;
   if (b > 148 * 32) b = 148 * 32;
@@ -260,6 +269,19 @@ static void launch_pure(Ctx& c, size_t smem, unsigned grid) {
   auto k = k_fused_pure<kMode, kU64>;
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k<<<grid, 512, smem, c.stream>>>(pure_params(c));
+}
+
+cudaError_t launch_need_tiles(Ctx& c) {
+  cudaError_t e;
+  if ((e = c.d_need.ensure((size_t)c.n_tiles + 1)) != cudaSuccess) return e;
+  if ((e = cudaMemsetAsync(c.d_need.p, 0, (size_t)c.n_tiles + 1, c.stream)) != cudaSuccess) return e;
+  const int64_t n = c.n_inside + c.n_isect;
+  if (n > 0) {
+    k_need_tiles<<<grid_for(n, 256), 256, 0, c.stream>>>(c.d_inside.as<int2>(), c.n_inside, c.d_isect.as<int2>(),
+                                                         c.n_isect, c.d_need.as<uint8_t>());
+    c.launches += 1;
+  }
+  return cudaGetLastError();
 }
 
 cudaError_t launch_fused(Ctx& c) {

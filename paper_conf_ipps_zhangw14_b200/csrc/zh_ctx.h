@@ -4,6 +4,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "zh_internal.cuh"
 
@@ -16,22 +17,27 @@
 
 namespace zh {
 
+// Process-wide cache of device blocks (zh_api.cu), like PyTorch's caching allocator: a context's
+// buffers go back to the cache when it is destroyed (after its streams are synchronised) and the
+// next context of the same device reuses them, so a zh_create / zh_run / zh_destroy cycle does not
+// pay cudaMalloc + cudaFree of a 40 GB raster copy every time.  zh_trim_cache() frees the cache.
+cudaError_t cache_alloc(void** p, size_t* got, size_t need);
+void cache_free(void* p, size_t bytes);
+
 // Grow-only device buffer owned by the context.
 struct DBuf {
   void* p = nullptr;
   size_t bytes = 0;
   cudaError_t ensure(size_t need) {
     if (need <= bytes && p) return cudaSuccess;
-    if (p) cudaFree(p);
+    if (p) cudaFree(p);  // growth: cudaFree waits for the work already enqueued on the old block
     p = nullptr;
     bytes = 0;
     if (need == 0) need = 16;
-    cudaError_t e = cudaMalloc(&p, need);
-    if (e == cudaSuccess) bytes = need;
-    return e;
+    return cache_alloc(&p, &bytes, need);
   }
-  void release() {
-    if (p) cudaFree(p);
+  void release() {  // callers have synchronised every stream that used the block
+    if (p) cache_free(p, bytes);
     p = nullptr;
     bytes = 0;
   }
@@ -85,6 +91,9 @@ struct Ctx {
   int64_t launches = 0;
   int64_t host_count_buf[4] = {0, 0, 0, 0};
   int64_t* pinned_counts = nullptr;
+  int64_t h2d_bytes = 0;               // bytes of raster copied host->device by the last upload
+  uint8_t* pinned_need = nullptr;       // on_host + fused zh_run: per-tile 'needed' flags (host copy)
+  DBuf d_need;
 };
 
 // kernels / launchers (k_*.cu)
@@ -101,6 +110,7 @@ size_t mixed_smem(Ctx& c);  // 0: the grouped cell kernel does not apply
 cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64_t grid, const int64_t* n_dev);
 cudaError_t launch_touch(Ctx& c, const int32_t* remap, cudaStream_t s);  // k_touch.cu (cover mode)
 cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
+cudaError_t launch_need_tiles(Ctx& c);  // d_need[t] = tile t has a pair (k_fused.cu)
 cudaError_t launch_zonal_stats(Ctx& c, int64_t* dstats);  // k_stats.cu
 cudaError_t launch_row_cost(Ctx& c, double* d_row_cost);  // k_fused.cu (shard planning)
 

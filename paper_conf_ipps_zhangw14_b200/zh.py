@@ -57,13 +57,14 @@ class zh_stats(ctypes.Structure):
     _fields_ = [("n_tiles", ctypes.c_int64), ("n_candidates", ctypes.c_int64), ("n_inside", ctypes.c_int64),
                 ("n_isect", ctypes.c_int64), ("n_band_entries", ctypes.c_int64), ("n_edges", ctypes.c_int64),
                 ("device_bytes", ctypes.c_int64), ("n_pure_tiles", ctypes.c_int64), ("n_pip_pairs", ctypes.c_int64),
-                ("n_pure_cells", ctypes.c_int64), ("n_pip_cells", ctypes.c_int64)]
+                ("n_pure_cells", ctypes.c_int64), ("n_pip_cells", ctypes.c_int64), ("h2d_bytes", ctypes.c_int64)]
 
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",
            "zh_fused_update", "zh_zonal_stats", "zh_plan_rows",
            "zh_run", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
-           "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy"]
+           "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy",
+           "zh_trim_cache", "zh_cache_bytes"]
 
 
 def _load():
@@ -97,6 +98,8 @@ def _load():
         "zh_last_error": (ctypes.c_char_p, []),
         "zh_abi_version": (i32, []),
         "zh_destroy": (None, [vp]),
+        "zh_trim_cache": (None, [i32]),
+        "zh_cache_bytes": (i64, []),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)

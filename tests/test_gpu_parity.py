@@ -244,6 +244,45 @@ def test_host_raster_path(tiny, cuda_device):
     assert (G == H).all()
 
 
+@pytest.mark.parametrize("tile", [100, 128])
+def test_host_raster_needed_tiles_only(tiny, cuda_device, tile):
+    """zh_run of the fused path on a HOST raster uploads only the tiles some pair needs (2-D copies of
+    tile runs, rounded out to 16-byte vectors; tiles not multiples of 8 wide; pitch > cols), and the
+    device copy outside them is never read: poisoned cached blocks and a poisoned pitch tail change
+    nothing."""
+    import torch
+    zh = _zh()
+    cfg, P, R, H = tiny
+    keep = [0, 5, 11, 15]  # a few polygons (15 = the enclave): most tiles have no pair
+    Ps = P.subset(keep)
+    pitch = cfg.cols + 24
+    host = np.full((cfg.rows, pitch), -7777, dtype=np.int16)
+    host[:, :cfg.cols] = R
+    pinned = torch.from_numpy(host).pin_memory()
+    # leave a poisoned block of the right size in libzh's cache: the context reuses it for its copy
+    with zh.ZonalHistogram(torch.full_like(pinned, 31000), cfg.gt, Ps, cfg.nbins, tile=tile, cols=cfg.cols,
+                           nodata=cfg.nodata, fused=False) as z:
+        z.run()
+    assert zh.LIB.zh_cache_bytes() > 0
+    for fused in (True, False):
+        with zh.ZonalHistogram(pinned, cfg.gt, Ps, cfg.nbins, tile=tile, cols=cfg.cols, nodata=cfg.nodata,
+                               fused=fused) as z:
+            G = z.run()
+            st = z.stats()
+        assert (G == H[keep]).all()
+        full = cfg.rows * pitch * 2
+        if fused:
+            assert 0 < st["h2d_bytes"] < full // 2, st["h2d_bytes"]
+        else:
+            assert st["h2d_bytes"] == full
+
+
+def test_cache_trim(cuda_device):
+    zh = _zh()
+    zh.LIB.zh_trim_cache(1)
+    assert zh.LIB.zh_cache_bytes() == 0
+
+
 def test_overlapping_polygons_and_linear_pattern(cuda_device):
     """Overlapping polygons count a cell in each; v = (r*cols + c) mod 4093 exercises all bins."""
     rows, cols = 512, 768
