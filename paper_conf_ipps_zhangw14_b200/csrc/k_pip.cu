@@ -69,15 +69,18 @@ __global__ void __launch_bounds__(kPipThreads, ZH_PIP_MINB) k_pip_cells(PipP p) 
 #ifndef ZH_MIX_THREADS
 #define ZH_MIX_THREADS 256
 #endif
+#ifndef ZH_MIX_CODE
+#define ZH_MIX_CODE 1  // k_mixed_cells: code-byte routing with B at a power-of-two offset (packed bins)
+#endif
 #ifndef ZH_MIX_MINB
 #define ZH_MIX_MINB 4
 #endif
 // Tile groups of <= 2 pairs (fused path): each cell read once per group (zh_pip.cuh).
-template <int kMode, bool kU64>
+template <int kMode, bool kU64, bool kCode>
 __global__ void __launch_bounds__(ZH_MIX_THREADS, ZH_MIX_MINB) k_mixed_cells(PipP p) {
   if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
   extern __shared__ __align__(16) uint32_t sh[];
-  mixed_cells_body<kMode, kU64>(p, blockIdx.x, sh);
+  mixed_cells_body<kMode, kU64, kCode>(p, blockIdx.x, sh);
 }
 
 cudaError_t launch_pip(Ctx& c) { return launch_pip_list(c, c.d_isect.as<int2>(), c.n_isect, nullptr); }
@@ -113,6 +116,8 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev) {
   if (p.rcc > c.rp.T) p.rcc = c.rp.T;
   p.pbits = c.d_pbits.as<uint32_t>();
   p.grp = nullptr;
+  p.offb = 0;
+  p.bmo = 0;
   return p;
 }
 
@@ -168,15 +173,37 @@ static int mixed_rows(const Ctx& c) {
   return std::max(1, std::min(c.rp.T, 1024 / wpo));
 }
 
-// Shared memory of k_mixed_cells, or 0 when the grouped form does not apply (two histograms must
-// fit the CTA, and the packed form needs 16-bit byte offsets over both).
+// Shared-memory layout of k_mixed_cells: histogram A at word 0, B at word *offb, the two staged
+// bitmaps at word *bmo.  With packed bins, B sits at a power of two (code bytes route the cells,
+// count8_fast_code) and the bitmaps fill the gap below it when they fit; otherwise B follows A.
+// Returns the bytes, or 0 when the grouped form does not apply (two histograms must fit the CTA,
+// and the packed forms need 16-bit byte offsets over both).
+static size_t mixed_layout(const Ctx& c, int* offb, int* bmo, bool* code) {
+  const int hw = hist_words(c.bp.nbins);
+  const int bmw = 2 * mixed_rows(c) * ((c.rp.T + 31) / 32);
+  const bool packed = pip_mode(c) >= 2;
+  int ob = 256;
+  while (ob < hw) ob *= 2;
+  const FastBins fb = make_fast_bins(c.bp);
+  const int nod_idx = 0xFFFF - (int)(fb.Cb2 & 0xFFFFu);
+  *code = ZH_MIX_CODE && packed && (ob + hw) * 4 < 65536 && (!fb.bias || nod_idx >= ob + hw);
+  if (*code) {
+    *offb = ob;
+    *bmo = (hw + bmw <= ob) ? hw : ob + hw;
+  } else {
+    *offb = hw;
+    *bmo = 2 * hw;
+  }
+  const size_t words = std::max<size_t>((size_t)*offb + hw, (size_t)*bmo + bmw);
+  if (words * 4 > 200 * 1024) return 0;
+  if (packed && !*code && 2 * (size_t)hw * 4 >= 65536) return 0;
+  return words * 4;
+}
 
 size_t mixed_smem(Ctx& c) {
-  const size_t hw = (size_t)hist_words(c.bp.nbins);
-  const size_t smem = 2 * hw * 4 + 2 * (size_t)mixed_rows(c) * ((c.rp.T + 31) / 32) * 4;
-  if (smem > 200 * 1024) return 0;
-  if (pip_mode(c) >= 2 && 2 * hw * 4 >= 65536) return 0;
-  return smem;
+  int ob, bo;
+  bool code;
+  return mixed_layout(c, &ob, &bo, &code);
 }
 
 cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64_t grid, const int64_t* n_dev) {
@@ -184,15 +211,19 @@ cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64
   PipP p = pip_params(c, pairs, n_dev);
   p.grp = grp;
   p.rcc = mixed_rows(c);
-  const size_t smem = mixed_smem(c);
+  bool code = false;
+  const size_t smem = mixed_layout(c, &p.offb, &p.bmo, &code);
   void (*k)(PipP);
+#define ZH_MIX_K(M) (c.out_u64 ? (code ? k_mixed_cells<M, true, true> : k_mixed_cells<M, true, false>) \
+                               : (code ? k_mixed_cells<M, false, true> : k_mixed_cells<M, false, false>))
   switch (pip_mode(c)) {
-    case 0: k = c.out_u64 ? k_mixed_cells<0, true> : k_mixed_cells<0, false>; break;
-    case 1: k = c.out_u64 ? k_mixed_cells<1, true> : k_mixed_cells<1, false>; break;
-    case 2: k = c.out_u64 ? k_mixed_cells<2, true> : k_mixed_cells<2, false>; break;
-    case 3: k = c.out_u64 ? k_mixed_cells<3, true> : k_mixed_cells<3, false>; break;
-    default: k = c.out_u64 ? k_mixed_cells<4, true> : k_mixed_cells<4, false>; break;
+    case 0: k = ZH_MIX_K(0); break;
+    case 1: k = ZH_MIX_K(1); break;
+    case 2: k = ZH_MIX_K(2); break;
+    case 3: k = ZH_MIX_K(3); break;
+    default: k = ZH_MIX_K(4); break;
   }
+#undef ZH_MIX_K
   if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k<<<(unsigned)grid, ZH_MIX_THREADS, smem, c.stream>>>(p);
   c.launches += 1;

@@ -233,6 +233,33 @@ __device__ __forceinline__ void count8_fast_sel(uint32_t* __restrict__ hist, con
   }
 }
 
+// Two histograms, A at word 0 and B at word `offb`, a power of two (>= 256) above every index of A:
+// a cell goes to B by OR-ing offb into its index.  One code byte per cell — 0 (A), offb >> 8 (B),
+// 0xFF (not counted) — lands in the high byte of the cell's 16-bit half (one PRMT per two cells);
+// the clamp to dumB2 = (offb + this lane's dummy slot) in both halves then sends not-counted cells
+// to B's dummy slots (never flushed).  The caller guarantees (offb + hist_words) * 4 < 2^16 and a
+// biased nodata index >= offb + hist_words.
+template <int kForm>
+__device__ __forceinline__ void count8_fast_code(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                                 uint32_t sel, const FastBins& f, uint32_t dumB2, uint32_t ob) {
+  const uint32_t e = sel & ~skip;
+  const uint32_t clo = (((skip & 0xFu) * 0x00204081u) & 0x01010101u) * 0xFFu +
+                       (((e & 0xFu) * 0x00204081u) & 0x01010101u) * ob;
+  const uint32_t chi = ((((skip >> 4) & 0xFu) * 0x00204081u) & 0x01010101u) * 0xFFu +
+                       ((((e >> 4) & 0xFu) * 0x00204081u) & 0x01010101u) * ob;
+  const uint32_t ws[4] = {q.x, q.y, q.z, q.w};
+  char* hb = reinterpret_cast<char*>(hist);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t j = (uint32_t)(i & 1) * 2;  // first of the two cells within its 4-cell code word
+    const uint32_t P = 4u | (j << 4) | (4u << 8) | ((j + 1) << 12);
+    uint32_t x = fast_idx2<kForm>(ws[i], f) | __byte_perm(i < 2 ? clo : chi, 0u, P);
+    x = __vminu2(x, dumB2) << 2;
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);
+  }
+}
+
 // Generic path (any width / lo / nbins): same layout, scalar mapping, per-cell atomics.
 template <bool kW1>
 __device__ __forceinline__ void count8_generic(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,

@@ -31,6 +31,8 @@ struct PipP {
   int wpo;               // words per stored parity row = ceil(T / 32)
   int rcc;               // rows per chunk of the split cell kernel's shared copy of the bitmap
   const int2* grp;       // tile groups of the cell kernel: {first pair index, #pairs (1 or 2)}
+  int offb;              // k_mixed_cells: word offset of the second histogram (B)
+  int bmo;               // k_mixed_cells: word offset of the two staged bitmaps
 };
 
 struct Ctx;  // zh_ctx.h
@@ -324,14 +326,17 @@ __device__ __forceinline__ void flush_hist(const uint32_t* __restrict__ hist, in
 // one atomic per cell, whatever m).  Otherwise (overlapping polygons, cover mode) every vector is
 // counted once per pair.  The branch is uniform over the CTA (__syncthreads_or of the overlap).
 // `sh` holds 2 hist_words(nbins) + 2 rcc * wpo words.
-template <int kMode, bool kU64>
+// kCode: B at a power-of-two offset, cells routed by code bytes (count8_fast_code); otherwise
+// count8_fast_sel / count8_generic_sel add the offset.
+template <int kMode, bool kU64, bool kCode>
 __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint32_t* __restrict__ sh) {
   const int HW = hist_words(p.bp.nbins);
   const int2 gr = p.grp[g];
   const int64_t pi0 = gr.x;
   const int m = gr.y;
+  const int OB = p.offb;
   uint32_t* hist = sh;
-  uint32_t* bm0 = sh + 2 * HW;
+  uint32_t* bm0 = sh + p.bmo;
   uint32_t* bm1 = bm0 + p.rcc * p.wpo;
   const RasterP& rp = p.rp;
   const int2 pr0 = p.isect[pi0];
@@ -345,11 +350,12 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
   const uint32_t* __restrict__ src0 = p.pbits + pi0 * (int64_t)rp.T * wpo;
   const uint32_t* __restrict__ src1 = src0 + (int64_t)rp.T * wpo;
 
-  for (int i = threadIdx.x * 4; i < m * HW; i += blockDim.x * 4)
-    *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
+  for (int i = threadIdx.x * 4; i < m * HW; i += blockDim.x * 4)  // A, then B
+    *reinterpret_cast<uint4*>(&hist[i < HW ? i : i - HW + OB]) = make_uint4(0, 0, 0, 0);
   const uint32_t dummy = (uint32_t)hist_dummy(p.bp.nbins) + (threadIdx.x & 31);
   const uint32_t dum2 = dummy * 0x10001u;
-  const uint32_t off2 = (uint32_t)HW * 0x10001u;
+  const uint32_t off2 = (uint32_t)OB * 0x10001u;
+  const uint32_t dumB2 = (dummy + (uint32_t)OB) * 0x10001u, ob = (uint32_t)OB >> 8;
   const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
   const int nk = (int)(k1 - k0);
   const int64_t pitch = rp.pitch;
@@ -359,8 +365,12 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
     else count8_generic<kMode == 0>(hh, q, skip, p.bp, dummy);
   };
   auto count_sel = [&](const uint4& q, uint32_t skip, uint32_t sel) {
-    if (kMode >= 2) count8_fast_sel<kMode - 2>(hist, q, skip, sel, fb, dum2, off2);
-    else count8_generic_sel<kMode == 0>(hist, q, skip, sel, p.bp, dummy, HW);
+    if constexpr (kMode >= 2) {
+      if (kCode) count8_fast_code<kMode - 2>(hist, q, skip, sel, fb, dumB2, ob);
+      else count8_fast_sel<kMode - 2>(hist, q, skip, sel, fb, dum2, off2);
+    } else {
+      count8_generic_sel<kMode == 0>(hist, q, skip, sel, p.bp, dummy, OB);
+    }
   };
 
   for (int cr = 0; cr < h; cr += p.rcc) {
@@ -446,7 +456,7 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
             if ((s0 & s1) == 0xFFu) continue;
             const uint4 q = ld_stream16(ptr);
             if (s0 != 0xFFu) count(q, s0, hist);
-            if (s1 != 0xFFu) count(q, s1, hist + HW);
+            if (s1 != 0xFFu) count(q, s1, hist + OB);
           }
         }
       };
@@ -469,14 +479,14 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
           if ((s0 & s1) == 0xFFu) continue;
           const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
           if (s0 != 0xFFu) count(q, s0, hist);
-          if (s1 != 0xFFu) count(q, s1, hist + HW);
+          if (s1 != 0xFFu) count(q, s1, hist + OB);
         }
       }
     }
     __syncthreads();
   }
   flush_hist<kU64>(hist, p.bp.nbins, kp0, p.out);
-  if (m > 1) flush_hist<kU64>(hist + HW, p.bp.nbins, kp1, p.out);
+  if (m > 1) flush_hist<kU64>(hist + OB, p.bp.nbins, kp1, p.out);
 }
 
 }  // namespace zh
