@@ -144,13 +144,17 @@ __device__ __forceinline__ void suffix_xor_store(const uint32_t* __restrict__ bm
     const uint32_t* row = bm + lr * wpr;
     uint32_t* orow = out + (int64_t)lr * wpo;
     uint32_t carry = 0;
+    // A row has one or two crossings, and neighbouring rows (the lanes of a warp) have theirs in the
+    // same word: words with no flip in any lane of the warp take the 1-op path (uniform branch).
+    const uint32_t lanes = __activemask();
     auto step = [&](uint32_t t) -> uint32_t {
+      if (!__any_sync(lanes, t != 0u)) return 0u - carry;
       t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
       const uint32_t v = (t >> 1) ^ (0u - carry);
       carry ^= (t & 1u);
       return v;
     };
-    for (int wi = wpr - 1; wi >= wpo; --wi) step(row[wi]);
+    for (int wi = wpr - 1; wi >= wpo; --wi) carry ^= __popc(row[wi]) & 1u;  // "all cells" flips: parity only
     if ((wpo & 3) == 0) {
       for (int g = wpo - 4; g >= 0; g -= 4) {
         uint4 v;
