@@ -146,6 +146,9 @@ typedef struct {
   int64_t n_pip_cells;    /* cells of the tiles of those pairs (counted once per pair)           */
   int64_t h2d_bytes;      /* on_host rasters: bytes copied host->device by the last zh_run /
                              zh_upload_raster                                                   */
+  int64_t n_mixed_groups; /* after zh_fused_update: tile groups (<= 2 pairs of one tile) of the
+                             grouped cell kernel (0 when it does not apply)                      */
+  int64_t n_group_cells;  /* cells those groups read (a mixed tile once per group)              */
 } zh_stats;
 
 /* Validate, copy polygons to the device (H2D on options->stream), allocate per-tile histograms

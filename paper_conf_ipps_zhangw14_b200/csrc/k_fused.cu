@@ -17,6 +17,10 @@
 #include "zh_pip.cuh"
 #include "zh_tilehist.cuh"
 
+#ifndef ZH_PURE_MINB
+#define ZH_PURE_MINB 3  // CTAs of 512 threads per SM the pure-tile kernel is compiled for (register cap)
+#endif
+
 #ifndef ZH_EXACT_GRID
 #define ZH_EXACT_GRID 1  // 1: step-4 grids sized from the list counts (host reads them during k_fused_pure)
 #endif
@@ -131,16 +135,23 @@ __global__ void k_pack_mixed(const uint32_t* __restrict__ cnt, int64_t n, uint64
   }
 }
 
-// grp[g] = {first pair index, #pairs}; counts[4] = #groups
+
+// grp[g] = {first pair index, #pairs}; counts[4] = #groups, counts[5] = cells read by the groups
+// (a mixed tile once per group: the grouped cell kernel's algorithmic bytes)
 __global__ void k_pip_groups(const uint32_t* __restrict__ cnt, const uint64_t* __restrict__ off, int64_t n_tiles,
-                             int2* __restrict__ grp, int64_t* __restrict__ counts) {
+                             RasterP rp, int2* __restrict__ grp, int64_t* __restrict__ counts) {
+  int64_t cells = 0;
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n_tiles; t += (int64_t)gridDim.x * blockDim.x) {
     const uint32_t c = cnt[t];
     if (!c) continue;
     const uint32_t p0 = (uint32_t)off[t], g0 = (uint32_t)(off[t] >> 32);
     for (uint32_t q = 0; 2 * q < c; ++q) grp[g0 + q] = make_int2((int)(p0 + 2 * q), (int)min(2u, c - 2 * q));
+    cells += tile_cells(rp, (int)t) * (int64_t)((c + 1) >> 1);
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) counts[4] = (int64_t)(off[n_tiles] >> 32);
+  for (int o = 16; o > 0; o >>= 1) cells += __shfl_xor_sync(0xffffffffu, cells, o);
+  if ((threadIdx.x & 31) == 0 && cells) atomicAdd(reinterpret_cast<unsigned long long*>(&counts[5]),
+                                                  (unsigned long long)cells);
 }
 
 struct PureP {
@@ -188,7 +199,7 @@ __device__ __forceinline__ void pure_tile_body(const PureP& f, int64_t idx, uint
 }
 
 template <int kMode, bool kU64>
-__global__ void __launch_bounds__(512, 3) k_fused_pure(PureP f) {
+__global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
   if ((int64_t)blockIdx.x >= f.counts[0]) return;
   extern __shared__ __align__(16) uint32_t sh[];
   pure_tile_body<kMode, kU64>(f, blockIdx.x, sh);
@@ -352,7 +363,7 @@ cudaError_t launch_fused(Ctx& c) {
   if (grouped) {
     if ((e = c.d_pip_grp.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
     k_pip_groups<<<grid_for(NT, 256), 256, 0, c.stream>>>(c.d_mixed.as<uint32_t>(), c.d_extra_pos.as<uint64_t>(), NT,
-                                                          c.d_pip_grp.as<int2>(), c.d_fcounts.as<int64_t>());
+                                                          c.rp, c.d_pip_grp.as<int2>(), c.d_fcounts.as<int64_t>());
     c.launches += 1;
   }
 

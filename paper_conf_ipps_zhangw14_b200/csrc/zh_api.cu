@@ -661,15 +661,17 @@ extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
   s->n_edges = c->V;
   s->device_bytes = (int64_t)zh::device_bytes(*c);
   s->h2d_bytes = c->h2d_bytes;
-  s->n_pure_tiles = s->n_pip_pairs = s->n_pure_cells = s->n_pip_cells = 0;
+  s->n_pure_tiles = s->n_pip_pairs = s->n_pure_cells = s->n_pip_cells = s->n_mixed_groups = s->n_group_cells = 0;
   if (c->fused_done) {
-    ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_fcounts.p, 4 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
+    ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
           "zh_get_stats");
     ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_stats");
     s->n_pure_tiles = c->pinned_counts[0];
     s->n_pip_pairs = c->pinned_counts[1];
     s->n_pure_cells = c->pinned_counts[2];
     s->n_pip_cells = c->pinned_counts[3];
+    s->n_mixed_groups = c->pinned_counts[4];
+    s->n_group_cells = c->pinned_counts[5];
   }
   return ZH_OK;
 }

@@ -11,6 +11,6 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 #    (step 1 four-step: k_tile_hist, k_aggregate, k_parity, k_pip_cells; step 2 fused: k_fused_pure,
 #    k_parity, k_pip_cells)
 timeout 900 ncu --set full --clock-control none --import-source on \
-    -k regex:"k_tile_hist|k_pip|k_aggregate|k_fused_pure|k_parity|k_touch" \
+    -k regex:"k_tile_hist|k_aggregate|k_parity|k_pip_cells|k_fused_pure|k_mixed_cells|k_touch" \
     -c 7 -o gpurun_out/full_${TAG} -f python tools/prof_step.py conus 256 2 four_fused > gpurun_out/full_${TAG}.log 2>&1
 echo profile done
