@@ -166,23 +166,26 @@ struct PureP {
   void* out;
 };
 
-// One pure tile: the step-1 shared histogram, added into each inside polygon's row.
-template <int kMode, bool kU64>
-__device__ __forceinline__ void pure_tile_body(const PureP& f, int64_t idx, uint32_t* __restrict__ sh) {
-  const int HW = hist_words(f.bp.nbins);
-  const int tile = f.pure_tiles[idx];
-  const int trl = tile / f.rp.TC, tc = tile - trl * f.rp.TC;
-  for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
-    *reinterpret_cast<uint4*>(&sh[i]) = make_uint4(0, 0, 0, 0);
-  __syncthreads();
-  tile_histogram<kMode>(sh, f.rp, f.bp, f.fb, trl, tc);
-  __syncthreads();
+// Same inside-polygon set for two pure tiles (lists compared in stored order: a permuted list only
+// costs an extra flush)?
+__device__ __forceinline__ bool same_polys(const PureP& f, int ta, int tb) {
+  const uint32_t ca = f.pure_cnt[ta];
+  if (ca != f.pure_cnt[tb]) return false;
+  const uint32_t a0 = (uint32_t)(f.pure_off[ta] & 0xFFFFFFFFull), b0 = (uint32_t)(f.pure_off[tb] & 0xFFFFFFFFull);
+  for (uint32_t j = 0; j < ca; ++j)
+    if (f.pure_poly[a0 + j] != f.pure_poly[b0 + j]) return false;
+  return true;
+}
+
+// Add the shared histogram into the row of each inside polygon of `tile` (one global atomic per
+// non-zero bin; 16-byte reads of the histogram skip whole zero vectors — a tile touches a few
+// hundred of 5,000 bins).
+template <bool kU64>
+__device__ __forceinline__ void pure_flush(const PureP& f, int tile, const uint32_t* __restrict__ sh) {
   const uint32_t beg = (uint32_t)(f.pure_off[tile] & 0xFFFFFFFFull), cnt = f.pure_cnt[tile];
   const int nbins = f.bp.nbins;
   for (uint32_t j = 0; j < cnt; ++j) {
     const int64_t row = (int64_t)f.pure_poly[beg + j] * nbins;
-    // 16-byte reads of the shared histogram (4 bins each); most tiles touch a few hundred of the
-    // 5,000 bins, so whole zero vectors are skipped with one test
     for (int b = threadIdx.x * 4; b < nbins; b += blockDim.x * 4) {
       const uint4 v = *reinterpret_cast<const uint4*>(&sh[kOff + b]);
       if (!(v.x | v.y | v.z | v.w)) continue;
@@ -198,11 +201,45 @@ __device__ __forceinline__ void pure_tile_body(const PureP& f, int64_t idx, uint
   }
 }
 
+// A CTA takes kPureRun consecutive entries of the pure-tile list (tile order: neighbouring tiles,
+// mostly of the same county) and keeps ONE shared histogram across consecutive tiles with the same
+// inside-polygon set: no barrier between them (the loads of the next tile follow the last atomics
+// of the previous one) and one flush per run instead of one per tile.
+#ifndef ZH_PURE_RUN
+#define ZH_PURE_RUN 8
+#endif
+constexpr int kPureRun = ZH_PURE_RUN;
+
 template <int kMode, bool kU64>
 __global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
-  if ((int64_t)blockIdx.x >= f.counts[0]) return;
+  const int64_t n = f.counts[0];
+  const int64_t i0 = (int64_t)blockIdx.x * kPureRun;
+  if (i0 >= n) return;
+  const int64_t i1 = min(n, i0 + (int64_t)kPureRun);
   extern __shared__ __align__(16) uint32_t sh[];
-  pure_tile_body<kMode, kU64>(f, blockIdx.x, sh);
+  const int HW = hist_words(f.bp.nbins);
+  auto zero = [&]() {
+    for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
+      *reinterpret_cast<uint4*>(&sh[i]) = make_uint4(0, 0, 0, 0);
+  };
+  zero();
+  __syncthreads();
+  int tile = f.pure_tiles[i0];
+  for (int64_t idx = i0; idx < i1; ++idx) {
+    const int trl = tile / f.rp.TC, tc = tile - trl * f.rp.TC;
+    tile_histogram<kMode>(sh, f.rp, f.bp, f.fb, trl, tc);
+    const int next = idx + 1 < i1 ? f.pure_tiles[idx + 1] : -1;
+    if (next < 0 || !same_polys(f, tile, next)) {  // uniform over the CTA
+      __syncthreads();
+      pure_flush<kU64>(f, tile, sh);
+      if (next >= 0) {
+        __syncthreads();
+        zero();
+        __syncthreads();
+      }
+    }
+    tile = next;
+  }
 }
 
 // ---- work-balanced shard planning: estimated cost of every tile row of the
@@ -406,7 +443,7 @@ cudaError_t launch_fused(Ctx& c) {
   if (c.timing) cudaEventRecord(c.ev[10], c.stream);
   if (NI > 0) {
     const size_t smem = (size_t)hist_words(c.bp.nbins) * 4;
-    const unsigned grid = (unsigned)NI;
+    const unsigned grid = (unsigned)((NI + kPureRun - 1) / kPureRun);
     if (c.out_u64) {
       switch (mode) {
         case 0: launch_pure<0, true>(c, smem, grid); break;
