@@ -49,7 +49,7 @@ __global__ void __launch_bounds__(256, ZH_PIP_MINB) k_pip(PipP p) {
 #define ZH_PAR_THREADS 128
 #endif
 #ifndef ZH_PAR_MINB
-#define ZH_PAR_MINB 12
+#define ZH_PAR_MINB 14
 #endif
 template <bool kRep>
 __global__ void __launch_bounds__(ZH_PAR_THREADS, ZH_PAR_MINB) k_parity(PipP p) {
