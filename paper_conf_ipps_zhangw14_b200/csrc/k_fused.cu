@@ -11,6 +11,8 @@
 //                           step-4 cell-in-polygon kernel, which is exact for any pair.
 // Each raster cell is therefore read once from HBM, and only when some polygon may contain it.
 // The result is bit-identical to steps 1 + 3 + 4 (integer sums; tests/test_gpu_fused.py).
+#include <algorithm>
+
 #include <cub/device/device_scan.cuh>
 
 #include "zh_ctx.h"
@@ -164,6 +166,7 @@ struct PureP {
   const uint32_t* pure_cnt;
   const int32_t* pure_poly;
   void* out;
+  int run;  // pure tiles per CTA (k_fused_pure)
 };
 
 // Same inside-polygon set for two pure tiles (lists compared in stored order: a permuted list only
@@ -201,10 +204,11 @@ __device__ __forceinline__ void pure_flush(const PureP& f, int tile, const uint3
   }
 }
 
-// A CTA takes kPureRun consecutive entries of the pure-tile list (tile order: neighbouring tiles,
-// mostly of the same county) and keeps ONE shared histogram across consecutive tiles with the same
-// inside-polygon set: no barrier between them (the loads of the next tile follow the last atomics
-// of the previous one) and one flush per run instead of one per tile.
+// A CTA takes f.run (<= ZH_PURE_RUN) consecutive entries of the pure-tile list (tile order:
+// neighbouring tiles, mostly of the same county) and keeps ONE shared histogram across consecutive
+// tiles with the same inside-polygon set: no barrier between them (the loads of the next tile
+// follow the last atomics of the previous one) and one flush per run instead of one per tile.
+// The host lowers the run when the list is short, so that the grid still fills the GPU.
 #ifndef ZH_PURE_RUN
 #define ZH_PURE_RUN 8
 #endif
@@ -213,9 +217,9 @@ constexpr int kPureRun = ZH_PURE_RUN;
 template <int kMode, bool kU64>
 __global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
   const int64_t n = f.counts[0];
-  const int64_t i0 = (int64_t)blockIdx.x * kPureRun;
+  const int64_t i0 = (int64_t)blockIdx.x * f.run;
   if (i0 >= n) return;
-  const int64_t i1 = min(n, i0 + (int64_t)kPureRun);
+  const int64_t i1 = min(n, i0 + (int64_t)f.run);
   extern __shared__ __align__(16) uint32_t sh[];
   const int HW = hist_words(f.bp.nbins);
   auto zero = [&]() {
@@ -309,6 +313,9 @@ static PureP pure_params(Ctx& c) {
   f.pure_cnt = c.d_pure_cnt.as<uint32_t>();
   f.pure_poly = c.d_pure_poly.as<int32_t>();
   f.out = c.d_out;
+  // enough CTAs for >= 4 waves of 3 per SM (148 SMs), at most kPureRun tiles each
+  int64_t run = c.n_inside / (148 * 3 * 4);
+  f.run = (int)std::max<int64_t>(1, std::min<int64_t>(kPureRun, run));
   return f;
 }
 
@@ -443,7 +450,8 @@ cudaError_t launch_fused(Ctx& c) {
   if (c.timing) cudaEventRecord(c.ev[10], c.stream);
   if (NI > 0) {
     const size_t smem = (size_t)hist_words(c.bp.nbins) * 4;
-    const unsigned grid = (unsigned)((NI + kPureRun - 1) / kPureRun);
+    const int run = pure_params(c).run;
+    const unsigned grid = (unsigned)((NI + run - 1) / run);
     if (c.out_u64) {
       switch (mode) {
         case 0: launch_pure<0, true>(c, smem, grid); break;
