@@ -42,7 +42,8 @@ __device__ __forceinline__ int64_t clamp_est(double v, int64_t lo, int64_t hi) {
 // Rows r in [rA, rB) with ya <= yc(r) < yb, exactly (monotone predicates + first_false).
 __device__ __forceinline__ int2 straddle_rows(const Geo& g, double ya, double yb, int64_t rA, int64_t rB) {
   if (!(ya < yb)) return make_int2(0, 0);
-  const double ea = (ya - g.gt3) / g.gt5 - g.oy, eb = (yb - g.gt3) / g.gt5 - g.oy;
+  // first guesses only (first_false makes the rows exact): reciprocal instead of a division
+  const double ea = (ya - g.gt3) * g.igt5 - g.oy, eb = (yb - g.gt3) * g.igt5 - g.oy;
   int64_t ra, rb;
   if (g.gt5 < 0) {  // yc decreasing in r
     // B(r): yc(r) < yb  is false then true -> ra = first r with B true
@@ -250,7 +251,7 @@ __global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges
     const Edge e = edges[v];
     const double xi = intercept(e, yc);
     // pred(j) = ((xc(c_j) < xi) == s), true on a prefix of j in [0, wk)
-    const double est = ((xi - g.gt0) / g.gt1 - g.ox) / rp.T - (double)m.x;
+    const double est = ((xi - g.gt0) * g.igt1 - g.ox) / rp.T - (double)m.x;  // a guess (first_false is exact)
     const int64_t jb = first_false(0, wk, clamp_est(est, 0, wk), [&](int64_t j) {
       return (col_centre(g, (int64_t)(m.x + j) * rp.T) < xi) == s;
     });

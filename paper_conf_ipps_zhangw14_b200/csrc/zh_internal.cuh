@@ -20,6 +20,7 @@ struct Geo {
   double gt0, gt1, gt3, gt5;
   double ox, oy;
   double igt1;  // 1 / gt1: only for first guesses of a column (every decision is exact, first_false)
+  double igt5;  // 1 / gt5: likewise for rows
 };
 
 // kRep = false: the centre (0.5 as an immediate — the hot kernels are instantiated for it, the
