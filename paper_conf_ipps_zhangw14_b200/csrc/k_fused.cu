@@ -313,9 +313,12 @@ static PureP pure_params(Ctx& c) {
   f.pure_cnt = c.d_pure_cnt.as<uint32_t>();
   f.pure_poly = c.d_pure_poly.as<int32_t>();
   f.out = c.d_out;
-  // enough CTAs for >= 4 waves of 3 per SM (148 SMs), at most kPureRun tiles each
-  int64_t run = c.n_inside / (148 * 3 * 4);
-  f.run = (int)std::max<int64_t>(1, std::min<int64_t>(kPureRun, run));
+  // enough CTAs for >= 4 waves of 3 per SM (148 SMs), at most kPureRun tiles of 256^2 cells each
+  // (more tiles when they are smaller: the zeroing and the flush are per run, not per cell)
+  const int64_t T2 = (int64_t)c.rp.T * c.rp.T;
+  const int64_t cap = std::max<int64_t>(kPureRun, std::min<int64_t>(256, kPureRun * 65536 / std::max<int64_t>(T2, 1)));
+  const int64_t run = c.n_inside / (148 * 3 * 4);
+  f.run = (int)std::max<int64_t>(1, std::min<int64_t>(cap, run));
   return f;
 }
 
