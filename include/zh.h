@@ -187,7 +187,9 @@ zh_status zh_run(zh_ctx ctx, void* host_out);
 
 /* Device memory of destroyed contexts is kept in a process-wide cache and reused by later
  * contexts of the same device (no cudaMalloc / cudaFree of the raster copy per zh_create /
- * zh_destroy cycle); allocations that fail return the cache to the driver and retry.
+ * zh_destroy cycle); allocations that fail return the cache to the driver and retry.  The
+ * contexts' small pinned host buffers are cached the same way (cudaFreeHost can stall for
+ * hundreds of ms while a large host raster is pinned).
  * zh_trim_cache frees every cached block; keep_caching = 0 also disables caching from then on.
  * zh_cache_bytes: bytes currently cached. */
 void zh_trim_cache(int32_t keep_caching);

@@ -59,7 +59,8 @@ BlockCache& cache() {
 void trim_locked(BlockCache& bc, int dev) {  // dev < 0: every device
   for (auto it = bc.free_blocks.begin(); it != bc.free_blocks.end();) {
     if (dev < 0 || it->second.first == dev) {
-      cudaFree(it->second.second);
+      if (it->second.first == -1) cudaFreeHost(it->second.second);
+      else cudaFree(it->second.second);
       bc.cached -= it->first;
       it = bc.free_blocks.erase(it);
     } else {
@@ -107,6 +108,39 @@ void zh::cache_free(void* p, size_t bytes) {
     return;
   }
   bc.free_blocks.emplace(bytes, std::make_pair(dev, p));
+  bc.cached += bytes;
+}
+
+// Small pinned host buffers (list sizes, needed-tile flags) go through the same cache (device key
+// -1): cudaFreeHost was measured taking 1 to 600 ms per call while a 40 GB host raster is pinned.
+static cudaError_t pinned_alloc(void** p, size_t* got, size_t need) {
+  BlockCache& bc = cache();
+  {
+    std::lock_guard<std::mutex> lk(bc.m);
+    for (auto it = bc.free_blocks.lower_bound(need); it != bc.free_blocks.end() && it->first <= 2 * need + 4096;
+         ++it) {
+      if (it->second.first != -1) continue;
+      *p = it->second.second;
+      *got = it->first;
+      bc.cached -= it->first;
+      bc.free_blocks.erase(it);
+      return cudaSuccess;
+    }
+  }
+  cudaError_t e = cudaHostAlloc(p, need, cudaHostAllocDefault);
+  if (e == cudaSuccess) *got = need;
+  return e;
+}
+
+static void pinned_free(void* p, size_t bytes) {
+  if (!p) return;
+  BlockCache& bc = cache();
+  std::lock_guard<std::mutex> lk(bc.m);
+  if (!bc.enabled) {
+    cudaFreeHost(p);
+    return;
+  }
+  bc.free_blocks.emplace(bytes, std::make_pair(-1, p));
   bc.cached += bytes;
 }
 
@@ -300,7 +334,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
     c->rp.data = c->raster_dev.as<int16_t>();
     if (r->pitch % 8 != 0) return cleanup_fail(fail(ZH_ERR_INVALID_ARG, "host raster pitch must be a multiple of 8"));
   }
-  if ((e = cudaHostAlloc((void**)&c->pinned_counts, 16 * sizeof(int64_t), cudaHostAllocDefault)) != cudaSuccess)
+  if ((e = pinned_alloc((void**)&c->pinned_counts, &c->pinned_counts_bytes, 16 * sizeof(int64_t))) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (pinned counters)"));
   for (int i = 0; i < 16; ++i)
     if ((e = cudaEventCreate(&c->ev[i])) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (events)"));
@@ -314,10 +348,24 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   return ZH_OK;
 }
 
+#ifdef ZH_DESTROY_TRACE
+#include <chrono>
+static double now_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+#define ZH_TR(label) fprintf(stderr, "zh_destroy %-10s %8.3f ms\n", label, now_ms() - t_tr), t_tr = now_ms()
+#else
+#define ZH_TR(label) (void)0
+#endif
+
 extern "C" void zh_destroy(zh_ctx h) {
   if (!h) return;
   Ctx* c = C(h);
+#ifdef ZH_DESTROY_TRACE
+  double t_tr = now_ms();
+#endif
   cudaStreamSynchronize(c->stream);
+  ZH_TR("sync");
   if (c->side) cudaStreamSynchronize(c->side);  // the blocks go back to the cache: nothing may still use them
   zh::DBuf* bufs[] = {&c->raster_dev, &c->d_pro, &c->d_rvo, &c->d_x, &c->d_y, &c->d_edges, &c->d_erows,
                       &c->d_mbb, &c->d_ncand, &c->d_nband, &c->d_cand_off,
@@ -328,8 +376,10 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats,
                       &c->d_pip_grp, &c->d_mixed_pk, &c->d_need};
   for (auto* b : bufs) b->release();
+  ZH_TR("release");
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  ZH_TR("events");
   if (c->side) {
     cudaStreamSynchronize(c->side);
     cudaStreamDestroy(c->side);
@@ -337,8 +387,10 @@ extern "C" void zh_destroy(zh_ctx h) {
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->ev_counts) cudaEventDestroy(c->ev_counts);
-  if (c->pinned_counts) cudaFreeHost(c->pinned_counts);
-  if (c->pinned_need) cudaFreeHost(c->pinned_need);
+  ZH_TR("streams");
+  pinned_free(c->pinned_counts, c->pinned_counts_bytes);
+  pinned_free(c->pinned_need, c->pinned_need_bytes);
+  ZH_TR("freehost");
   delete c;
 }
 
@@ -382,7 +434,7 @@ static zh_status upload_needed(Ctx* c) {
   const int64_t NT = c->n_tiles, T = c->rp.T, TC = c->rp.TC;
   c->h2d_bytes = 0;
   if (NT == 0 || c->rp.nrows == 0) return ZH_OK;
-  if (!c->pinned_need) ZH_CU(cudaHostAlloc((void**)&c->pinned_need, (size_t)NT + 1, cudaHostAllocDefault), "zh_run");
+  if (!c->pinned_need) ZH_CU(pinned_alloc((void**)&c->pinned_need, &c->pinned_need_bytes, (size_t)NT + 1), "zh_run");
   ZH_CU(zh::launch_need_tiles(*c), "zh_run (needed tiles)");
   ZH_CU(cudaMemcpyAsync(c->pinned_need, c->d_need.p, (size_t)NT, cudaMemcpyDeviceToHost, c->stream), "zh_run");
   ZH_CU(cudaStreamSynchronize(c->stream), "zh_run (needed tiles)");

@@ -93,6 +93,7 @@ struct Ctx {
   int64_t* pinned_counts = nullptr;
   int64_t h2d_bytes = 0;               // bytes of raster copied host->device by the last upload
   uint8_t* pinned_need = nullptr;       // on_host + fused zh_run: per-tile 'needed' flags (host copy)
+  size_t pinned_counts_bytes = 0, pinned_need_bytes = 0;  // sizes of the cached pinned blocks
   DBuf d_need;
 };
 
