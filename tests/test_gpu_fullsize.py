@@ -1,13 +1,13 @@
 """Full-size GPU parity (BASELINE.json state-scale and CONUS-scale configs, the bench's launch
 configuration): sampled per-polygon histograms vs the oracle (computed one polygon at a time on
-the polygon's raster window), plus properties that hold at any size — tile-size invariance,
+the polygon's raster window; BASELINE.json configs [1], [2] and [4]), plus properties that hold at any size — tile-size invariance,
 force-all-intersect invariance, and (state tiling covers the extent) the partition identity
 sum_k H_k == global histogram of the mapped raster."""
 import numpy as np
 import pytest
 
 import oracle
-from synth.configs import CONUS, STATE
+from synth.configs import CONUS, PIPSTRESS, STATE
 from synth.dem import fill_device, fill_host
 
 pytestmark = pytest.mark.gpu
@@ -91,4 +91,31 @@ def test_conus_full_size(cuda_device):
     G2, _ = _run(t, cfg, P, tile=360)  # the paper's 0.1 degree tile
     assert (G2 == G).all()
     # every counted cell is a real, non-nodata cell
+    assert G.sum() <= cfg.cells
+
+
+def test_pipstress_full_size(cuda_device):
+    """BASELINE.json configs[4]: the CONUS raster with 50k small jagged polygons (mostly
+    intersecting tiles) over the tile-size sweep.  Fused and four-step paths at T = 256; the fused
+    path alone at T = 64 (the four-step path would need 98.8 GB of tile histograms)
+    and T = 1024 (no inside tile at all).  Every tile size gives the same histograms; sampled
+    polygons equal the oracle."""
+    import torch
+    from paper_conf_ipps_zhangw14_b200 import zh
+    cfg = PIPSTRESS
+    P = cfg.polygons()
+    t = _raster(cfg)
+    G, st = _run(t, cfg, P)
+    assert st["n_isect"] > 10 * st["n_inside"] > 0
+    for k in _sample_polys(P, 8, 3):
+        assert (G[k] == _oracle_poly(cfg, P, k)).all(), k
+    torch.cuda.empty_cache()
+    for tile in (64, 1024):
+        with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=tile, cols=cfg.cols, nodata=cfg.nodata,
+                               fused=True) as z:
+            Gt = z.run()
+            if tile == 1024:
+                assert z.stats()["n_inside"] == 0
+        assert (Gt == G).all(), tile
+        torch.cuda.empty_cache()
     assert G.sum() <= cfg.cells
