@@ -210,6 +210,8 @@ def main():
                          "testing the cell centre (not the headline configuration)")
     ap.add_argument("--equal-shards", action="store_true",
                     help="N > 1: equal tile-row strips instead of the work-balanced plan (zh_plan_rows)")
+    ap.add_argument("--dense-reduce", action="store_true",
+                    help="N > 1: NCCL reduce of all n_poly rows instead of the sparse reduce (dist.SparseReducer)")
     args = ap.parse_args()
 
     from synth.configs import CONFIGS
@@ -225,7 +227,7 @@ def main():
     import torch.distributed as dist
 
     from paper_conf_ipps_zhangw14_b200 import zh
-    from paper_conf_ipps_zhangw14_b200.dist import plan_shards, reduce_histograms
+    from paper_conf_ipps_zhangw14_b200.dist import SparseReducer, plan_shards, reduce_histograms, touched_polygons
     from synth.dem import fill_device
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -267,6 +269,21 @@ def main():
                           fused=(args.path == "fused"), cover=args.cover)
     z.set_output(out)
 
+    # N > 1: sparse reduce (only polygons spanning strips are summed; the plan is geometry only),
+    # unless --dense-reduce or the shared-GPU gloo mode (gloo has no CUDA point-to-point)
+    reducer = None
+    if world > 1 and not args.dense_reduce and not shared:
+        z.zh_pair_tiles()
+        reducer = SparseReducer(touched_polygons(z), P.n_poly, device=out.device)
+        log(f"sparse reduce: {len(reducer.shared)} shared polygons, {reducer.rows_moved()} rows moved "
+            f"(dense: {world * P.n_poly})")
+
+    def reduce_out():
+        if reducer is not None:
+            reducer.reduce(out, to_rank0=True)
+        else:
+            reduce_histograms(out, to_rank0=True)  # only rank 0 reads the result (half the traffic of an all-reduce)
+
     path = args.path
     z.set_timing(True)
     lib_ms = []  # per timed step: the library's own event timings (steps, fused inner kernels)
@@ -283,7 +300,7 @@ def main():
         if record:
             lib_ms.append(z.step_ms())  # syncs after the step's last kernel
         if world > 1:
-            reduce_histograms(out, to_rank0=True)  # only rank 0 reads the result (half the traffic of an all-reduce)
+            reduce_out()
 
     clk = ClockSampler(local).__enter__()
     time.sleep(0.5)  # nvidia-smi needs a moment before its first sample
@@ -388,7 +405,7 @@ def main():
     e2e = None
     host = None
     if not args.no_e2e:
-        e2e, host = run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log)
+        e2e, host = run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log, reduce_out)
     z.close()
 
     cpu = None
@@ -411,7 +428,8 @@ def main():
                 "data": "synthetic (fractal int16 DEM + jagged Voronoi counties, seeded)",
                 "config": dict(cfg.describe(), n_poly=P.n_poly, n_vert=P.n_vert,
                                parallelism=f"tile-row shards x{world}" + (" (shared GPU, gloo)" if shared else "")
-                               + ("" if world == 1 else (" equal" if args.equal_shards else " work-balanced")),
+                               + ("" if world == 1 else (" equal" if args.equal_shards else " work-balanced"))
+                               + ("" if world == 1 else (" sparse-reduce" if reducer is not None else " dense-reduce")),
                                l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA",
                                semantics="closed rectangle meets polygon (R15)" if args.cover else "centre inside"),
                 "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
@@ -426,14 +444,13 @@ def main():
     return 0
 
 
-def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log):
+def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log, reduce_out):
     """E2E through the public API: host raster (pinned) + host polygons -> host histogram."""
     import numpy as np
     import torch
     import torch.distributed as dist
 
     from paper_conf_ipps_zhangw14_b200 import zh
-    from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms
 
     # pinned host copy of this rank's strip (identical to the device one; D2H is not timed)
     host = np.empty((max(nrows, 1), pitch), dtype=np.int16)
@@ -459,7 +476,7 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
         if world > 1:
             z2.set_output(out)
             z2.zh_run(None)
-            reduce_histograms(out, to_rank0=True)  # only rank 0 reads the result (half the traffic of an all-reduce)
+            reduce_out()
             if rank == 0:
                 res_pin.copy_(out, non_blocking=True)
             torch.cuda.synchronize()

@@ -46,3 +46,107 @@ def reduce_histograms(out, group=None, to_rank0: bool = False):
     else:
         dist.all_reduce(out, op=dist.ReduceOp.SUM, group=group)
     return out
+
+
+def sparse_plan(touched):
+    """Who sends what ('a sparse reduce of only the polygons that span shards').
+
+    touched[r, k] — rank r's partial histogram of polygon k may be non-zero (every k with a step-2
+    pair in r's strip; any superset is correct).  Returns (shared, owned): `shared` = polygons
+    touched by >= 2 ranks (summed with a collective over their rows only); owned[r] = polygons
+    touched by rank r alone (their rows are already final on r and are only moved, not summed).
+    Polygons touched by no rank stay zero everywhere.  Pure host logic, same on every rank."""
+    import numpy as np
+    t = np.asarray(touched, dtype=bool)
+    n = t.sum(axis=0)
+    shared = np.nonzero(n >= 2)[0].astype(np.int64)
+    owned = [np.nonzero((n == 1) & t[r])[0].astype(np.int64) for r in range(t.shape[0])]
+    return shared, owned
+
+
+def touched_polygons(z) -> "np.ndarray":
+    """Polygons with a step-2 pair (inside or intersecting) in the strip of context `z` (after
+    zh_pair_tiles): the only rows of its partial histogram that can be non-zero."""
+    import numpy as np
+    ins, isx = z.pairs_host()
+    return np.unique(np.concatenate([ins[:, 1], isx[:, 1]])).astype(np.int64)
+
+
+class SparseReducer:
+    """Sum per-rank partial histograms moving only rows that can be non-zero.
+
+    The plan is geometry only (built once per decomposition from each rank's touched polygons and
+    one all-gather of P-byte masks).  Per call: the rows of polygons that span strips are packed
+    and reduced (to rank 0) or all-reduced; the rows of single-strip polygons are final on their
+    rank and are sent to rank 0 (point-to-point), or all-gathered for the all-reduce form.  With
+    tile-row strips only the polygons crossing a strip border are summed, and every other row
+    crosses the fabric at most once (the dense NCCL reduce moves all n_poly rows through every
+    link).  Integer sums: bit-identical to `reduce_histograms` (tests/test_dist.py)."""
+
+    def __init__(self, touched, n_poly: int, group=None, device=None):
+        import numpy as np
+        import torch
+        import torch.distributed as dist
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        mask = torch.zeros(n_poly, dtype=torch.uint8)
+        mask[torch.as_tensor(np.asarray(touched, dtype=np.int64))] = 1
+        mask = mask.to(device) if device is not None else mask
+        masks = [torch.empty_like(mask) for _ in range(self.world)]
+        dist.all_gather(masks, mask, group=group)
+        self.shared, self.owned = sparse_plan(torch.stack(masks).cpu().numpy())
+        dev = mask.device
+        self._shared = torch.as_tensor(self.shared, device=dev)
+        self._owned = [torch.as_tensor(o, device=dev) for o in self.owned]
+        self.max_owned = max(len(o) for o in self.owned)
+
+    def rows_moved(self) -> int:
+        """Rows each call puts on the fabric (reduce form): shared rows once per rank + owned rows
+        of ranks != 0."""
+        return len(self.shared) * self.world + sum(len(o) for o in self.owned[1:])
+
+    def reduce(self, out, to_rank0: bool = False):
+        import torch
+        import torch.distributed as dist
+        if self.world == 1:
+            return out
+        g = self.group
+        if len(self.shared):
+            buf = out.index_select(0, self._shared)
+            if to_rank0:
+                dist.reduce(buf, dst=dist.get_global_rank(g, 0) if g is not None else 0, group=g)
+            else:
+                dist.all_reduce(buf, group=g)
+            if not to_rank0 or self.rank == 0:
+                out.index_copy_(0, self._shared, buf)
+        if to_rank0:
+            ops, bufs = [], []
+            glob = (lambda r: dist.get_global_rank(g, r)) if g is not None else (lambda r: r)
+            if self.rank == 0:
+                for r in range(1, self.world):
+                    if len(self.owned[r]):
+                        b = torch.empty((len(self.owned[r]), out.shape[1]), dtype=out.dtype, device=out.device)
+                        bufs.append((r, b))
+                        ops.append(dist.P2POp(dist.irecv, b, glob(r), g))
+            elif len(self.owned[self.rank]):
+                b = out.index_select(0, self._owned[self.rank])
+                bufs.append((self.rank, b))
+                ops.append(dist.P2POp(dist.isend, b, glob(0), g))
+            if ops:
+                for w in dist.batch_isend_irecv(ops):
+                    w.wait()
+            if self.rank == 0:
+                for r, b in bufs:
+                    out.index_copy_(0, self._owned[r], b)
+        elif self.max_owned:
+            mine = self._owned[self.rank]
+            send = torch.zeros((self.max_owned, out.shape[1]), dtype=out.dtype, device=out.device)
+            if len(mine):
+                send[:len(mine)] = out.index_select(0, mine)
+            recv = torch.empty((self.world * self.max_owned, out.shape[1]), dtype=out.dtype, device=out.device)
+            dist.all_gather_into_tensor(recv, send, group=g)
+            for r in range(self.world):
+                if r != self.rank and len(self.owned[r]):
+                    out.index_copy_(0, self._owned[r], recv[r * self.max_owned:r * self.max_owned + len(self.owned[r])])
+        return out

@@ -85,3 +85,73 @@ def test_gloo_world2_reduce_equals_single_process():
     for r in range(world):
         assert (res[r][0] == H).all()
     assert (res[0][1] == H).all()
+
+
+def test_sparse_plan_host_logic():
+    from paper_conf_ipps_zhangw14_b200.dist import sparse_plan
+    t = np.array([[1, 1, 0, 0, 1],
+                  [0, 1, 1, 0, 0],
+                  [0, 1, 0, 0, 1]], bool)
+    shared, owned = sparse_plan(t)
+    assert shared.tolist() == [1, 4]
+    assert [o.tolist() for o in owned] == [[0], [2], []]
+    # every touched polygon is either shared or owned by exactly one rank; untouched ones by none
+    cover = np.zeros(5, int)
+    cover[shared] += 1
+    for o in owned:
+        cover[o] += 1
+    assert cover.tolist() == [1, 1, 1, 0, 1]
+
+
+def _sparse_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_ipps_zhangw14_b200.dist import SparseReducer
+        from synth.configs import TINY as cfg
+        from synth.dem import fill_host
+        P = cfg.polygons()
+        r0, r1 = shard_rows(cfg.rows, cfg.tile, world, rank)
+        R = fill_host(cfg.dem, cfg.cols, r0, 0, r1 - r0, cfg.cols, nthreads=2)
+        H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata), row0=r0, nthreads=2)
+        # touched = the rows that can be non-zero, plus a few spurious ones (any superset is valid)
+        extra = np.random.default_rng(rank).integers(0, P.n_poly, 2)
+        touched = np.union1d(np.nonzero(H.any(axis=1))[0], extra)
+        red = SparseReducer(touched, P.n_poly)
+        t = torch.from_numpy(H.view(np.int64).copy())
+        t0 = t.clone()
+        red.reduce(t)                   # all-reduce form
+        red.reduce(t0, to_rank0=True)   # reduce form
+        red.reduce(torch.from_numpy(H.view(np.int64).copy()), to_rank0=True)  # reusable plan
+        q.put((rank, (t.numpy().view(np.uint64).copy(), t0.numpy().view(np.uint64).copy(),
+                      len(red.shared), red.rows_moved())))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_sparse_reduce_equals_single_process(world):
+    import oracle
+    from synth.configs import TINY as cfg
+    from synth.dem import fill_host
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sparse_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    P = cfg.polygons()
+    R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata))
+    for r in range(world):
+        assert (res[r][0] == H).all()
+    assert (res[0][1] == H).all()
+    n_shared = res[0][2]
+    assert 0 < n_shared < P.n_poly  # some polygons span the strip borders, not all
+    assert res[0][3] < world * P.n_poly  # fewer rows on the fabric than the dense reduce

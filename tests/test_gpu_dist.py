@@ -1,7 +1,9 @@
 """The multi-GPU path on one GPU: world_size 2 processes (torch.distributed, gloo over the same
 cuda:0 — there is one GPU in this environment), each holding a tile-row strip of the tiny and
 state rasters in HBM, running libzh on its strip (both paths), and all-reducing the int64 view of
-the uint64 histograms.  The reduced result must equal the oracle bit for bit."""
+the uint64 histograms.  The reduced result must equal the oracle bit for bit — also through the
+sparse reduce (dist.SparseReducer, on host copies: gloo has no CUDA point-to-point), whose plan
+comes from the touched polygons of libzh's step-2 pairs (every non-zero row must be touched)."""
 import os
 import socket
 
@@ -24,7 +26,7 @@ def _worker(rank, world, port, cfg_name, q):
     import torch.distributed as dist
 
     from paper_conf_ipps_zhangw14_b200 import zh
-    from paper_conf_ipps_zhangw14_b200.dist import reduce_histograms, shard_rows
+    from paper_conf_ipps_zhangw14_b200.dist import SparseReducer, reduce_histograms, shard_rows, touched_polygons
     from synth.configs import CONFIGS
     from synth.dem import fill_device
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -46,9 +48,15 @@ def _worker(rank, world, port, cfg_name, q):
                                    row0=r0, nodata=cfg.nodata, fused=fused) as z:
                 z.set_output(out)
                 z.zh_run(None)
+                touched = touched_polygons(z)
+            part = out.cpu()
+            nz = np.nonzero(part.numpy().any(axis=1))[0]
+            assert np.isin(nz, touched).all()
             reduce_histograms(out, to_rank0=fused)  # four-step: all-reduce; fused: reduce to rank 0 (bench.py)
             res.append(out.cpu().numpy().view(np.uint64).copy())
-        q.put((rank, res[0], res[1]))
+        SparseReducer(touched, P.n_poly).reduce(part, to_rank0=True)
+        res.append(part.numpy().view(np.uint64).copy())
+        q.put((rank, res[0], res[1], res[2]))
     finally:
         dist.destroy_process_group()
 
@@ -85,11 +93,14 @@ def test_two_ranks_reduce_to_oracle(cuda_device, cfg_name):
             r0, r1, c0, c1 = oracle.polygon_window(P, k, cfg.gt, cfg.rows, cfg.cols)
             win = fill_host(cfg.dem, cfg.cols, r0, c0, r1 - r0, c1 - c0)
             want[k] = oracle.o1(win, cfg.gt, P.subset([k]), bins, row0=r0, col0=c0)[0]
-    for rank, four, fused in got:
+    for rank, four, fused, sparse in got:
         for k in rows:
             assert (four[k] == want[k]).all(), (rank, k)
             if rank == 0:
                 assert (fused[k] == want[k]).all(), (rank, k)
+                assert (sparse[k] == want[k]).all(), (rank, k)
+        if rank == 0:
+            assert (sparse == fused).all()
 
 
 def test_plan_rows_balanced_shards(cuda_device):
