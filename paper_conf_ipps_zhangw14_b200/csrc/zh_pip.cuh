@@ -7,6 +7,11 @@
 #ifndef ZH_MIX_ROWS4
 #define ZH_MIX_ROWS4 1
 #endif
+// k_mixed_cells: the two staged parity bitmaps interleaved word by word ({A word, B word} pairs), so
+// that one 8-byte shared load gives a vector's bits of both pairs.
+#ifndef ZH_MIX_IL
+#define ZH_MIX_IL 1
+#endif
 
 namespace zh {
 
@@ -319,6 +324,23 @@ __device__ __forceinline__ void flush_hist(const uint32_t* __restrict__ hist, in
   }
 }
 
+// bits8 of both interleaved bitmaps: row = {A, B} word pairs of one bitmap row (wpr words each).
+__device__ __forceinline__ uint2 bits8_il(const uint2* __restrict__ row, int wpr, int lc0) {
+  if (lc0 >= 0) {
+    const int wi = lc0 >> 5, sh = lc0 & 31;
+    const uint2 a = row[wi];
+    uint64_t v0 = a.x, v1 = a.y;
+    if (sh > 24 && wi + 1 < wpr) {
+      const uint2 b = row[wi + 1];
+      v0 |= (uint64_t)b.x << 32;
+      v1 |= (uint64_t)b.y << 32;
+    }
+    return make_uint2((uint32_t)(v0 >> sh) & 0xFFu, (uint32_t)(v1 >> sh) & 0xFFu);
+  }
+  const uint2 a = row[0];
+  return make_uint2((a.x << (-lc0)) & 0xFFu, (a.y << (-lc0)) & 0xFFu);
+}
+
 // Cells of a GROUP of pairs of one mixed tile (p.grp[g] = {first pair index, m}, m = 1 or 2; the
 // pair list is grouped by tile), with the parity bitmaps of k_parity: each 16-byte vector is read
 // ONCE for both pairs.  When no cell of the tile is inside both polygons (always, for polygons that
@@ -382,8 +404,13 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
       for (int i = threadIdx.x; i < ch * wpo / 4; i += blockDim.x) {
         const uint4 a = __ldcs(s0 + i);
         const uint4 b = m > 1 ? __ldcs(s1 + i) : make_uint4(0, 0, 0, 0);
+#if ZH_MIX_IL
+        reinterpret_cast<uint4*>(bm0)[2 * i] = make_uint4(a.x, b.x, a.y, b.y);
+        reinterpret_cast<uint4*>(bm0)[2 * i + 1] = make_uint4(a.z, b.z, a.w, b.w);
+#else
         reinterpret_cast<uint4*>(bm0)[i] = a;
         reinterpret_cast<uint4*>(bm1)[i] = b;
+#endif
         ov |= (a.x & b.x) | (a.y & b.y) | (a.z & b.z) | (a.w & b.w);
       }
     } else {
@@ -391,8 +418,12 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
       const uint32_t* s1 = src1 + (int64_t)cr * wpo;
       for (int i = threadIdx.x; i < ch * wpo; i += blockDim.x) {
         const uint32_t a = __ldcs(s0 + i), b = m > 1 ? __ldcs(s1 + i) : 0u;
+#if ZH_MIX_IL
+        reinterpret_cast<uint2*>(bm0)[i] = make_uint2(a, b);
+#else
         bm0[i] = a;
         bm1[i] = b;
+#endif
         ov |= a & b;
       }
     }
@@ -408,9 +439,19 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
         const uint32_t cskip = cols_skip8(cs, c0, w);
         const int lc0 = (int)(cs - c0);
         const int wi = lc0 >> 5, bsh = lc0 & 31;
-        auto pbits = [&](const uint32_t* bm, int lr) -> uint32_t {
-          if (kA) return (bm[lr * wpo + wi] >> bsh) & 0xFFu;
-          return bits8(bm + lr * wpo, wpo, lc0);
+        // {bits of pair A, bits of pair B} of this thread's vector in local row lr
+        auto pb2 = [&](int lr) -> uint2 {
+#if ZH_MIX_IL
+          const uint2* row = reinterpret_cast<const uint2*>(bm0) + lr * wpo;
+          if (kA) {
+            const uint2 v = row[wi];
+            return make_uint2((v.x >> bsh) & 0xFFu, (v.y >> bsh) & 0xFFu);
+          }
+          return bits8_il(row, wpo, lc0);
+#else
+          if (kA) return make_uint2((bm0[lr * wpo + wi] >> bsh) & 0xFFu, (bm1[lr * wpo + wi] >> bsh) & 0xFFu);
+          return make_uint2(bits8(bm0 + lr * wpo, wpo, lc0), bits8(bm1 + lr * wpo, wpo, lc0));
+#endif
         };
         const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
         const int64_t step = (int64_t)rpi * pitch;
@@ -423,8 +464,9 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
             uint4 q[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
-              e[u] = pbits(bm1, lr + u * rpi);
-              s[u] = cskip | (~(pbits(bm0, lr + u * rpi) | e[u]) & 0xFFu);
+              const uint2 b2 = pb2(lr + u * rpi);
+              e[u] = b2.y;
+              s[u] = cskip | (~(b2.x | b2.y) & 0xFFu);
               q[u] = make_uint4(0, 0, 0, 0);
               if (s[u] != 0xFFu) q[u] = ld_stream16(ptr + u * step);
             }
@@ -434,9 +476,10 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
           }
 #endif
           for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
-            const uint32_t e0 = pbits(bm1, lr), e1 = pbits(bm1, lr + rpi);
-            const uint32_t s0 = cskip | (~(pbits(bm0, lr) | e0) & 0xFFu);
-            const uint32_t s1 = cskip | (~(pbits(bm0, lr + rpi) | e1) & 0xFFu);
+            const uint2 b0 = pb2(lr), b1 = pb2(lr + rpi);
+            const uint32_t e0 = b0.y, e1 = b1.y;
+            const uint32_t s0 = cskip | (~(b0.x | e0) & 0xFFu);
+            const uint32_t s1 = cskip | (~(b1.x | e1) & 0xFFu);
             uint4 q0 = make_uint4(0, 0, 0, 0), q1 = make_uint4(0, 0, 0, 0);
             if (s0 != 0xFFu) q0 = ld_stream16(ptr);
             if (s1 != 0xFFu) q1 = ld_stream16(ptr + step);
@@ -444,15 +487,17 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
             if (s1 != 0xFFu) count_sel(q1, s1, e1);
           }
           for (; lr < ch; lr += rpi, ptr += step) {
-            const uint32_t e = pbits(bm1, lr);
-            const uint32_t skip = cskip | (~(pbits(bm0, lr) | e) & 0xFFu);
+            const uint2 b2 = pb2(lr);
+            const uint32_t e = b2.y;
+            const uint32_t skip = cskip | (~(b2.x | e) & 0xFFu);
             if (skip == 0xFFu) continue;
             count_sel(ld_stream16(ptr), skip, e);
           }
         } else {
           for (; lr < ch; lr += rpi, ptr += step) {
-            const uint32_t s0 = cskip | (~pbits(bm0, lr) & 0xFFu);
-            const uint32_t s1 = cskip | (~pbits(bm1, lr) & 0xFFu);
+            const uint2 b2 = pb2(lr);
+            const uint32_t s0 = cskip | (~b2.x & 0xFFu);
+            const uint32_t s1 = cskip | (~b2.y & 0xFFu);
             if ((s0 & s1) == 0xFFu) continue;
             const uint4 q = ld_stream16(ptr);
             if (s0 != 0xFFu) count(q, s0, hist);
@@ -474,8 +519,13 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
         for (int kk = threadIdx.x; kk < nk; kk += blockDim.x) {
           const int64_t cs = (k0 + kk) * 8;
           const uint32_t cskip = cols_skip8(cs, c0, w);
-          const uint32_t s0 = cskip | (~bits8(bm0 + lr * wpo, wpo, (int)(cs - c0)) & 0xFFu);
-          const uint32_t s1 = cskip | (~bits8(bm1 + lr * wpo, wpo, (int)(cs - c0)) & 0xFFu);
+#if ZH_MIX_IL
+          const uint2 b2 = bits8_il(reinterpret_cast<const uint2*>(bm0) + lr * wpo, wpo, (int)(cs - c0));
+#else
+          const uint2 b2 = make_uint2(bits8(bm0 + lr * wpo, wpo, (int)(cs - c0)), bits8(bm1 + lr * wpo, wpo, (int)(cs - c0)));
+#endif
+          const uint32_t s0 = cskip | (~b2.x & 0xFFu);
+          const uint32_t s1 = cskip | (~b2.y & 0xFFu);
           if ((s0 & s1) == 0xFFu) continue;
           const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
           if (s0 != 0xFFu) count(q, s0, hist);
