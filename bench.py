@@ -459,6 +459,14 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
     reg = cudart.cudaHostRegister(host.ctypes.data, nbytes, 0)
     pinned = int(reg) == 0 if not isinstance(reg, tuple) else int(reg[0]) == 0
     torch.from_numpy(host)[:nrows].copy_(raster_v)
+    # the polygon vertex arrays are pinned too (zh_create's H2D of 154 MB then runs at PCIe speed
+    # instead of through pageable staging)
+    poly_pinned = []
+    for a in (P.x, P.y):
+        if a.flags.c_contiguous and a.dtype == np.float64 and a.nbytes:
+            rv = cudart.cudaHostRegister(a.ctypes.data, a.nbytes, 0)
+            if (int(rv) if not isinstance(rv, tuple) else int(rv[0])) == 0:
+                poly_pinned.append(a)
     torch.cuda.synchronize()
     z.close()  # free the resident context's tile histograms before the e2e context allocates its own
     res_pin = torch.empty((P.n_poly, cfg.nbins), dtype=torch.int64, pin_memory=True)
@@ -492,6 +500,8 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
             times.append(float(t.item()))
     if pinned:
         cudart.cudaHostUnregister(host.ctypes.data)
+    for a in poly_pinned:
+        cudart.cudaHostUnregister(a.ctypes.data)
     host = host[:nrows, :cfg.cols]
     sec = sum(times) / len(times)
     poly_bytes = P.x.nbytes + P.y.nbytes + P.poly_ring_off.nbytes // 2 + P.ring_vert_off.nbytes // 2
@@ -503,7 +513,7 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
     d2h = P.n_poly * cfg.nbins * 8
     log(f"e2e {sec:.3f} s/step (pinned={pinned})")
     return {"value": cfg.cells / sec, "unit": "cells/s", "seconds_per_step": sec, "h2d_bytes_per_step": h2d,
-            "d2h_bytes_per_step": d2h, "host_raster_pinned": bool(pinned), "steps": len(times),
+            "d2h_bytes_per_step": d2h, "host_raster_pinned": bool(pinned), "host_vertices_pinned": len(poly_pinned) == 2, "steps": len(times),
             "raster_h2d_bytes": raster_h2d, "raster_bytes": nrows * pitch * 2,
             "includes": f"zh_create (polygon H2D, allocation from libzh's block cache) + zh_run ({args.path}: step 2, "
                         f"raster H2D of the tiles some pair needs, steps) + result D2H + zh_destroy"}, host
