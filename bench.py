@@ -300,8 +300,16 @@ def main():
         if record:
             lib_ms.append(z.step_ms())  # syncs after the step's last kernel
         if world > 1:
-            reduce_out()
+            if record:
+                r0e, r1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                r0e.record(stream)
+                reduce_out()
+                r1e.record(stream)
+                red_ev.append((r0e, r1e))
+            else:
+                reduce_out()
 
+    red_ev = []  # per timed step: events around the histogram reduction (N > 1)
     clk = ClockSampler(local).__enter__()
     time.sleep(0.5)  # nvidia-smi needs a moment before its first sample
     for _ in range(args.warmup):
@@ -361,6 +369,11 @@ def main():
     if path == "fused":
         # the parity bitmaps of the mixed pairs (FP64 crossing work; after k_fused_pure, exact grid)
         steps_detail["k_parity"] = {"ms": avg(lib_ms, "fused_parity_kernel")}
+    if red_ev:
+        steps_detail["reduce_histograms"] = {
+            "ms": sum(a.elapsed_time(b) for a, b in red_ev) / len(red_ev),
+            "kind": "sparse" if reducer is not None else "dense",
+            "rows_moved": reducer.rows_moved() if reducer is not None else world * P.n_poly}
     dom = max(kern, key=lambda k: kern[k][0] or 0.0)
     dom_ms, dom_b = kern[dom]
     achieved = dom_b / (dom_ms / 1000.0) / 1e9
