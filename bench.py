@@ -270,9 +270,9 @@ def main():
     z.set_output(out)
 
     # N > 1: sparse reduce (only polygons spanning strips are summed; the plan is geometry only),
-    # unless --dense-reduce or the shared-GPU gloo mode (gloo has no CUDA point-to-point)
+    # unless --dense-reduce (the shared-GPU gloo mode stages its point-to-point rows through the host)
     reducer = None
-    if world > 1 and not args.dense_reduce and not shared:
+    if world > 1 and not args.dense_reduce:
         z.zh_pair_tiles()
         reducer = SparseReducer(touched_polygons(z), P.n_poly, device=out.device)
         log(f"sparse reduce: {len(reducer.shared)} shared polygons, {reducer.rows_moved()} rows moved "
@@ -378,7 +378,9 @@ def main():
     dom_ms, dom_b = kern[dom]
     achieved = dom_b / (dom_ms / 1000.0) / 1e9
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic_from_profile(dom),
+                "frac": achieved / peaks["hbm_gbs"],
+                # the ncu capture is of the N = 1 launch; a shard's launch is a different one
+                "traffic": traffic_from_profile(dom) if world == 1 else None,
                 "peak_source": peaks["source"], "alg_bytes_per_launch": dom_b,
                 "share_of_step": dom_ms / ms if ms > 0 else None}
     log(f"timed ({path}): {ms:.3f} ms/step, {steps_detail}")

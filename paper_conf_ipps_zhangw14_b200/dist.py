@@ -92,11 +92,12 @@ class SparseReducer:
         self.rank = dist.get_rank(group)
         mask = torch.zeros(n_poly, dtype=torch.uint8)
         mask[torch.as_tensor(np.asarray(touched, dtype=np.int64))] = 1
-        mask = mask.to(device) if device is not None else mask
+        if device is not None and dist.get_backend(group) != "gloo":
+            mask = mask.to(device)
         masks = [torch.empty_like(mask) for _ in range(self.world)]
         dist.all_gather(masks, mask, group=group)
         self.shared, self.owned = sparse_plan(torch.stack(masks).cpu().numpy())
-        dev = mask.device
+        dev = torch.device(device) if device is not None else mask.device
         self._shared = torch.as_tensor(self.shared, device=dev)
         self._owned = [torch.as_tensor(o, device=dev) for o in self.owned]
         self.max_owned = max(len(o) for o in self.owned)
@@ -120,17 +121,20 @@ class SparseReducer:
                 dist.all_reduce(buf, group=g)
             if not to_rank0 or self.rank == 0:
                 out.index_copy_(0, self._shared, buf)
+        # gloo has no CUDA point-to-point / all-gather-into-tensor: stage those rows through host
+        # memory (the shared-GPU test mode); NCCL moves them device to device
+        dev = torch.device("cpu") if out.is_cuda and dist.get_backend(g) == "gloo" else out.device
         if to_rank0:
             ops, bufs = [], []
             glob = (lambda r: dist.get_global_rank(g, r)) if g is not None else (lambda r: r)
             if self.rank == 0:
                 for r in range(1, self.world):
                     if len(self.owned[r]):
-                        b = torch.empty((len(self.owned[r]), out.shape[1]), dtype=out.dtype, device=out.device)
+                        b = torch.empty((len(self.owned[r]), out.shape[1]), dtype=out.dtype, device=dev)
                         bufs.append((r, b))
                         ops.append(dist.P2POp(dist.irecv, b, glob(r), g))
             elif len(self.owned[self.rank]):
-                b = out.index_select(0, self._owned[self.rank])
+                b = out.index_select(0, self._owned[self.rank]).to(dev)
                 bufs.append((self.rank, b))
                 ops.append(dist.P2POp(dist.isend, b, glob(0), g))
             if ops:
@@ -138,15 +142,16 @@ class SparseReducer:
                     w.wait()
             if self.rank == 0:
                 for r, b in bufs:
-                    out.index_copy_(0, self._owned[r], b)
+                    out.index_copy_(0, self._owned[r], b.to(out.device))
         elif self.max_owned:
             mine = self._owned[self.rank]
-            send = torch.zeros((self.max_owned, out.shape[1]), dtype=out.dtype, device=out.device)
+            send = torch.zeros((self.max_owned, out.shape[1]), dtype=out.dtype, device=dev)
             if len(mine):
-                send[:len(mine)] = out.index_select(0, mine)
-            recv = torch.empty((self.world * self.max_owned, out.shape[1]), dtype=out.dtype, device=out.device)
+                send[:len(mine)] = out.index_select(0, mine).to(dev)
+            recv = torch.empty((self.world * self.max_owned, out.shape[1]), dtype=out.dtype, device=dev)
             dist.all_gather_into_tensor(recv, send, group=g)
             for r in range(self.world):
                 if r != self.rank and len(self.owned[r]):
-                    out.index_copy_(0, self._owned[r], recv[r * self.max_owned:r * self.max_owned + len(self.owned[r])])
+                    rows = recv[r * self.max_owned:r * self.max_owned + len(self.owned[r])]
+                    out.index_copy_(0, self._owned[r], rows.to(out.device))
         return out

@@ -54,9 +54,13 @@ def _worker(rank, world, port, cfg_name, q):
             assert np.isin(nz, touched).all()
             reduce_histograms(out, to_rank0=fused)  # four-step: all-reduce; fused: reduce to rank 0 (bench.py)
             res.append(out.cpu().numpy().view(np.uint64).copy())
+        part_dev = part.cuda()
         SparseReducer(touched, P.n_poly).reduce(part, to_rank0=True)
         res.append(part.numpy().view(np.uint64).copy())
-        q.put((rank, res[0], res[1], res[2]))
+        # the same on the device tensor (what bench.py does; gloo stages the point-to-point rows)
+        SparseReducer(touched, P.n_poly, device=part_dev.device).reduce(part_dev, to_rank0=True)
+        res.append(part_dev.cpu().numpy().view(np.uint64).copy())
+        q.put((rank, res[0], res[1], res[2], res[3]))
     finally:
         dist.destroy_process_group()
 
@@ -93,7 +97,7 @@ def test_two_ranks_reduce_to_oracle(cuda_device, cfg_name):
             r0, r1, c0, c1 = oracle.polygon_window(P, k, cfg.gt, cfg.rows, cfg.cols)
             win = fill_host(cfg.dem, cfg.cols, r0, c0, r1 - r0, c1 - c0)
             want[k] = oracle.o1(win, cfg.gt, P.subset([k]), bins, row0=r0, col0=c0)[0]
-    for rank, four, fused, sparse in got:
+    for rank, four, fused, sparse, sparse_dev in got:
         for k in rows:
             assert (four[k] == want[k]).all(), (rank, k)
             if rank == 0:
@@ -101,6 +105,7 @@ def test_two_ranks_reduce_to_oracle(cuda_device, cfg_name):
                 assert (sparse[k] == want[k]).all(), (rank, k)
         if rank == 0:
             assert (sparse == fused).all()
+            assert (sparse_dev == fused).all()
 
 
 def test_plan_rows_balanced_shards(cuda_device):
