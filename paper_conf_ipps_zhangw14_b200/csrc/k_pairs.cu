@@ -22,6 +22,10 @@
 
 #include "zh_ctx.h"
 
+#ifndef ZH_MARK_RCP
+#define ZH_MARK_RCP 1
+#endif
+
 namespace zh {
 
 __device__ __forceinline__ int64_t upper_bound_i64(const int64_t* a, int64_t n, int64_t v) {
@@ -206,9 +210,16 @@ __global__ void __launch_bounds__(256) k_mark(const int32_t* __restrict__ pro, c
   const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
   for (int v = vb + threadIdx.x; v < ve; v += blockDim.x) {
     const Edge e = edges[v];
+    // fractional cell coordinates of the edge's bbox: reciprocals instead of divisions (a few ulp
+    // of a coordinate, far inside the one-cell margin below)
+#if ZH_MARK_RCP
+    double ca = (fmin(e.xa, e.xb) - g.gt0) * g.igt1, cb = (fmax(e.xa, e.xb) - g.gt0) * g.igt1;
+    double ra = (e.ya - g.gt3) * g.igt5, rb = (e.yb - g.gt3) * g.igt5;
+#else
     double ca = (fmin(e.xa, e.xb) - g.gt0) / g.gt1, cb = (fmax(e.xa, e.xb) - g.gt0) / g.gt1;
-    if (ca > cb) { double t = ca; ca = cb; cb = t; }
     double ra = (e.ya - g.gt3) / g.gt5, rb = (e.yb - g.gt3) / g.gt5;
+#endif
+    if (ca > cb) { double t = ca; ca = cb; cb = t; }
     if (ra > rb) { double t = ra; ra = rb; rb = t; }
     const double clo = fmax(floor(ca) - 1.0, (double)m.x * rp.T);
     const double chi = fmin(floor(cb) + 1.0, (double)(m.y + 1) * rp.T - 1.0);
