@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 5
+#define ZH_ABI_VERSION 6
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -104,7 +104,8 @@ typedef struct {
  * no check):  a cell with use_nodata && v == nodata is never counted; otherwise
  * d = v - lo; d < 0 -> bin 0 (clamp) or not counted (oor_drop); b = d / width;
  * b >= nbins -> nbins-1 (clamp) or not counted (oor_drop).
- * Requires 1 <= nbins <= 49152 (shared-memory histograms), 1 <= width, |lo| <= 1<<30. */
+ * Requires 1 <= nbins <= 49152 (shared-memory histograms), 1 <= width, |lo| <= 1<<30, and, with
+ * use_nodata, -32768 <= nodata <= 32767 (an int16 value; else INVALID_ARG). */
 typedef struct {
   int32_t lo, width, nbins;
   int32_t use_nodata, nodata;
@@ -112,8 +113,9 @@ typedef struct {
 } zh_bins;
 
 typedef struct {
-  int32_t tile;        /* T >= 1, arbitrary ("allow users to set it arbitrarily");
-                          partial edge tiles hold only real cells                                */
+  int32_t tile;        /* 1 <= T <= 46340, arbitrary ("allow users to set it
+                          arbitrarily"); partial edge tiles hold only real cells; T > 46340 ->
+                          UNSUPPORTED (per-tile counts are uint32: T^2 < 2^31)                   */
   int32_t out_u64;     /* 1: uint64 output (default); 0: uint32 (ZH_ERR_OVERFLOW at zh_create if
                           some polygon's MBB could hold >= 2^32 cells)                           */
   int32_t force_isect; /* 1: classify every non-outside pair as intersecting (skips step 3's
@@ -206,6 +208,45 @@ int64_t zh_cache_bytes(void);
  * NULL) a BORROWED device pointer. */
 #define ZH_NSTATS 8
 zh_status zh_zonal_stats(zh_ctx ctx, int64_t* host_stats, int64_t** dptr);
+
+/* Zonal summary in value units (the "min, max, average, count and standard deviation" of
+ * PAPER.md:10 §I ¶1), derived on the device from zh_zonal_stats' exact integers n = count,
+ * S1 = sum_b b*H[b], S2 = sum_b b^2*H[b].  A bin stands for the value lo + b*width (its lower
+ * edge: the cell value itself for width = 1 and unclamped cells; R16).  Per polygon
+ * ZH_NSUMMARY doubles, every step ONE correctly rounded binary64 operation (bit-reproducible):
+ *   [0] count = n
+ *   [1] min, [2] max, [3] lower median = lo + b*width for the bins of zh_zonal_stats (exact)
+ *   [4] mean = lo + width * (S1 / n)                         (RN of: S1 -> double, /, *, +)
+ *   [5] std  = width * (sqrt(D) / n), D = n*S2 - S1^2         (population standard deviation;
+ *            D exact in 128 bits, then RN of: D -> double, sqrt, /, *)
+ * [1]..[5] are NaN for an empty polygon.  Requires every count < 2^40.  Needs a completed
+ * histogram (as zh_zonal_stats).  host_out (n_poly * ZH_NSUMMARY, may be NULL) receives a copy
+ * (syncs); *dptr (may be NULL) a BORROWED device pointer. */
+#define ZH_NSUMMARY 6
+zh_status zh_zonal_summary(zh_ctx ctx, double* host_out, double** dptr);
+
+/* Histogram feature distances (§I ¶1: the per-zone histograms "can further be used
+ * as feature vectors for ... computing various distance measurements which can be used for
+ * subsequent clustering").  Between the NORMALISED histograms p = H_a / n_a, q = H_b / n_b of
+ * polygons a and b (n = count):
+ *   ZH_DIST_L1   sum_b |p_b - q_b|                       = RN(RN(RN(N) / n_a) / n_b),
+ *                N = sum_b |H_a[b]*n_b - H_b[b]*n_a|  (an exact 128-bit integer: bit-exact)
+ *   ZH_DIST_EMD  sum_b |P_b - Q_b|, P, Q the cumulative distributions (1-D earth mover's
+ *                distance in bin units; times width for value units); same form with the
+ *                cumulative counts C_a[b] = sum_{b' <= b} H_a[b'] in place of H (bit-exact)
+ *   ZH_DIST_CHI2 1/2 sum_{b: p_b + q_b > 0} (p_b - q_b)^2 / (p_b + q_b), evaluated as
+ *                0.5 * RN(RN(sum_b RN(RN(d^2) / s)) / n_a) / n_b) with d = RN(|H_a[b] n_b - H_b[b] n_a|),
+ *                s = RN(H_a[b] n_b + H_b[b] n_a), the sum in an unspecified order: relative
+ *                error <= (nbins + 8) * 2^-53
+ * NaN when either polygon is empty.  a_ids, b_ids: HOST int32 arrays of n polygon ids (each in
+ * [0, n_poly), else INVALID_ARG); host_out[i] = d(a_ids[i], b_ids[i]).  a_ids = b_ids = NULL:
+ * ALL pairs, host_out is [n_poly][n_poly] row-major (n ignored), symmetric, zero diagonal for
+ * non-empty polygons.  Needs a completed histogram (as zh_zonal_stats).  Syncs. */
+#define ZH_DIST_L1 0
+#define ZH_DIST_EMD 1
+#define ZH_DIST_CHI2 2
+zh_status zh_hist_distance(zh_ctx ctx, int32_t kind, const int32_t* a_ids, const int32_t* b_ids, int64_t n,
+                           double* host_out);
 
 /* Work-balanced multi-GPU decomposition (the paper's future work on load
  * balancing across nodes, §IV.C): split the raster's rows into n_shards contiguous

@@ -120,14 +120,16 @@ def crossings(P, k: int, xc: float, yc: float) -> int:
                                   x.ctypes.data, y.ctypes.data))
 
 
-def _hist(fn, win, row0, col0, gt, P, bins, nthreads, extra, rep=None):
+def _hist(fn, win, row0, col0, gt, P, bins, nthreads, extra, rep=None, out=None):
     win = np.asarray(win)
     assert win.dtype == np.int16 and win.ndim == 2 and win.strides[1] == 2
     nrows, ncols = win.shape
     pitch = win.strides[0] // 2
     g = _gt8(gt, rep)
     pro, rvo, x, y = _poly_args(P)
-    out = np.zeros((P.n_poly, bins.nbins), dtype=np.uint64)
+    if out is None:
+        out = np.zeros((P.n_poly, bins.nbins), dtype=np.uint64)
+    assert out.dtype == np.uint64 and out.shape == (P.n_poly, bins.nbins) and out.flags.c_contiguous
     fn(win.ctypes.data, int(row0), int(col0), nrows, ncols, pitch, g.ctypes.data, P.n_poly,
        pro.ctypes.data, rvo.ctypes.data, x.ctypes.data, y.ctypes.data, ctypes.byref(bins), out.ctypes.data,
        *extra, _nthreads(nthreads))
@@ -140,9 +142,11 @@ def o0(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, prefilter: bool = F
     return _hist(_L().zho_o0, win, row0, col0, gt, P, bins, nthreads, (int(prefilter),), rep)
 
 
-def o1(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, nthreads=None, rep=None):
-    """O1: row-hoisted intercepts, identical comparisons to O0.  Returns uint64 [n_poly, nbins]."""
-    return _hist(_L().zho_o1, win, row0, col0, gt, P, bins, nthreads, (), rep)
+def o1(win, gt, P, bins: Bins, row0: int = 0, col0: int = 0, nthreads=None, rep=None, out=None):
+    """O1: row-hoisted intercepts, identical comparisons to O0.  Returns uint64 [n_poly, nbins]
+    (accumulated into `out` when given: rows are independent, so bands of a raster can be fed
+    one after another)."""
+    return _hist(_L().zho_o1, win, row0, col0, gt, P, bins, nthreads, (), rep, out)
 
 
 def seg_touches(x0, y0, x1, y1, X0, X1, Y0, Y1) -> bool:

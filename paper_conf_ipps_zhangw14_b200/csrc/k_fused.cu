@@ -318,7 +318,9 @@ static PureP pure_params(Ctx& c) {
   const int64_t T2 = (int64_t)c.rp.T * c.rp.T;
   const int64_t cap = std::max<int64_t>(kPureRun, std::min<int64_t>(256, kPureRun * 65536 / std::max<int64_t>(T2, 1)));
   const int64_t run = c.n_inside / (148 * 3 * 4);
-  f.run = (int)std::max<int64_t>(1, std::min<int64_t>(cap, run));
+  // the shared uint32 histogram is kept across a run of tiles: run * T^2 < 2^32 (zh_create caps T)
+  const int64_t no_wrap = std::max<int64_t>(1, (int64_t)0xFFFFFFFFll / std::max<int64_t>(T2, 1));
+  f.run = (int)std::max<int64_t>(1, std::min<int64_t>(std::min<int64_t>(cap, run), no_wrap));
   return f;
 }
 

@@ -3,6 +3,7 @@
 #include <math.h>
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -189,6 +190,11 @@ static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bin
   if (b->nbins < 1 || b->nbins > kMaxBins) return fail(ZH_ERR_INVALID_ARG, "nbins must be in [1, %d]", kMaxBins);
   if (b->width < 1) return fail(ZH_ERR_INVALID_ARG, "width must be >= 1");
   if (b->lo > (1 << 30) || b->lo < -(1 << 30)) return fail(ZH_ERR_INVALID_ARG, "|lo| must be <= 2^30");
+  if (b->use_nodata && (b->nodata < -32768 || b->nodata > 32767))
+    return fail(ZH_ERR_INVALID_ARG, "nodata (%d) is not an int16 value", (int)b->nodata);
+  // per-tile / per-pair shared histograms and the pure-run accumulator count in uint32: a tile must
+  // hold < 2^32 cells, and the pure kernel caps its run of tiles accordingly (pure_params)
+  if (o->tile > 46340) return fail(ZH_ERR_UNSUPPORTED, "tile size > 46340 (T^2 must stay below 2^31 cells)");
   if (p->n_poly < 0 || p->n_ring < 0 || p->n_vert < 0) return fail(ZH_ERR_INVALID_ARG, "negative polygon counts");
   if (p->n_vert >= (1ll << 31) - 1 || p->n_ring >= (1ll << 31) - 1 || p->n_poly >= (1ll << 31) - 1)
     return fail(ZH_ERR_UNSUPPORTED, "more than 2^31 vertices/rings/polygons");
@@ -344,6 +350,9 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
       (e = cudaEventCreateWithFlags(&c->ev_counts, cudaEventDisableTiming)) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (side stream)"));
   if ((e = cudaGetLastError()) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
+  // the polygon arrays are the caller's (zh.h: they may be freed or reused once zh_create
+  // returns); with page-locked host arrays the copies above are truly asynchronous
+  if ((e = cudaStreamSynchronize(c->stream)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (H2D)"));
   *out = reinterpret_cast<zh_ctx>(c);
   return ZH_OK;
 }
@@ -374,7 +383,7 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
                       &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats,
-                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_need};
+                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
   for (auto* b : bufs) b->release();
   ZH_TR("release");
   for (int i = 0; i < 16; ++i)
@@ -402,7 +411,7 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
                             &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats,
-                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_need};
+                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;
@@ -580,8 +589,8 @@ extern "C" zh_status zh_run(zh_ctx h, void* host_out) {
 extern "C" zh_status zh_zonal_stats(zh_ctx h, int64_t* host_stats, int64_t** dptr) {
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
-  if (!c->have_pairs || !(c->fused_done || c->step4_done))
-    return fail(ZH_ERR_STATE, "zh_zonal_stats needs a completed histogram (zh_run or steps 2 + 3/4 or fused)");
+  if (!c->have_pairs || !(c->fused_done || (c->step3_done && c->step4_done)))
+    return fail(ZH_ERR_STATE, "zh_zonal_stats needs a completed histogram (zh_run, steps 2 + 3 + 4, or the fused update)");
   ZH_CU(c->d_stats.ensure((size_t)(c->P > 0 ? c->P : 1) * ZH_NSTATS * sizeof(int64_t)), "zh_zonal_stats");
   ZH_CU(zh::launch_zonal_stats(*c, c->d_stats.as<int64_t>()), "zh_zonal_stats");
   if (dptr) *dptr = c->d_stats.as<int64_t>();
@@ -591,6 +600,85 @@ extern "C" zh_status zh_zonal_stats(zh_ctx h, int64_t* host_stats, int64_t** dpt
           "zh_zonal_stats (D2H)");
     ZH_CU(cudaStreamSynchronize(c->stream), "zh_zonal_stats");
   }
+  return ZH_OK;
+}
+
+// Exact statistics of the current histogram into c->d_stats (a completed histogram required).
+static zh_status stats_on_device(Ctx* c, const char* who) {
+  if (!c->have_pairs || !(c->fused_done || (c->step3_done && c->step4_done)))
+    return fail(ZH_ERR_STATE, "%s needs a completed histogram (zh_run, steps 2 + 3 + 4, or the fused update)", who);
+  ZH_CU(c->d_stats.ensure((size_t)(c->P > 0 ? c->P : 1) * ZH_NSTATS * sizeof(int64_t)), who);
+  ZH_CU(zh::launch_zonal_stats(*c, c->d_stats.as<int64_t>()), who);
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_zonal_summary(zh_ctx h, double* host_out, double** dptr) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  zh_status s = stats_on_device(c, "zh_zonal_summary");
+  if (s != ZH_OK) return s;
+  ZH_CU(c->d_summary.ensure((size_t)(c->P > 0 ? c->P : 1) * ZH_NSUMMARY * sizeof(double)), "zh_zonal_summary");
+  ZH_CU(zh::launch_zonal_summary(*c, c->d_stats.as<int64_t>(), c->d_summary.as<double>()), "zh_zonal_summary");
+  if (dptr) *dptr = c->d_summary.as<double>();
+  if (host_out && c->P > 0) {
+    ZH_CU(cudaMemcpyAsync(host_out, c->d_summary.p, (size_t)c->P * ZH_NSUMMARY * sizeof(double),
+                          cudaMemcpyDeviceToHost, c->stream),
+          "zh_zonal_summary (D2H)");
+    ZH_CU(cudaStreamSynchronize(c->stream), "zh_zonal_summary");
+  }
+  return ZH_OK;
+}
+
+extern "C" zh_status zh_hist_distance(zh_ctx h, int32_t kind, const int32_t* a_ids, const int32_t* b_ids, int64_t n,
+                                      double* host_out) {
+  if (!h || !host_out) return fail(ZH_ERR_INVALID_ARG, "null argument");
+  Ctx* c = C(h);
+  if (kind != ZH_DIST_L1 && kind != ZH_DIST_EMD && kind != ZH_DIST_CHI2)
+    return fail(ZH_ERR_INVALID_ARG, "unknown distance kind %d", (int)kind);
+  if ((a_ids == nullptr) != (b_ids == nullptr))
+    return fail(ZH_ERR_INVALID_ARG, "a_ids and b_ids must both be given or both be NULL");
+  const bool all = a_ids == nullptr;
+  if (!all) {
+    if (n < 0 || n >= (1ll << 31)) return fail(ZH_ERR_INVALID_ARG, "n must be in [0, 2^31)");
+    for (int64_t i = 0; i < n; ++i)
+      if (a_ids[i] < 0 || a_ids[i] >= c->P || b_ids[i] < 0 || b_ids[i] >= c->P)
+        return fail(ZH_ERR_INVALID_ARG, "polygon id out of range at %lld", (long long)i);
+  } else if ((int64_t)c->P * c->P >= (1ll << 40)) {
+    return fail(ZH_ERR_UNSUPPORTED, "all-pairs matrix too large");
+  }
+  zh_status s = stats_on_device(c, "zh_hist_distance");
+  if (s != ZH_OK) return s;
+  // 32 x 32 -> 64-bit products when every count (and so every bin and running sum) is < 2^32
+  std::vector<int64_t> st((size_t)std::max(c->P, 1) * ZH_NSTATS);
+  if (c->P > 0) {
+    ZH_CU(cudaMemcpyAsync(st.data(), c->d_stats.p, st.size() * 8, cudaMemcpyDeviceToHost, c->stream), "zh_hist_distance");
+    ZH_CU(cudaStreamSynchronize(c->stream), "zh_hist_distance");
+  }
+  // ZH_DIST_WIDE=1 (testing): the general 64 x 64 -> 128-bit products even when narrow would do
+  const char* wide_env = getenv("ZH_DIST_WIDE");
+  bool narrow = !(wide_env && wide_env[0] == '1');
+  for (int32_t k = 0; k < c->P; ++k)
+    if ((uint64_t)st[(size_t)k * ZH_NSTATS] >= (1ull << 32)) narrow = false;
+  const int64_t n_out = all ? (int64_t)c->P * c->P : n;
+  ZH_CU(c->d_dist.ensure((size_t)std::max<int64_t>(n_out, 1) * sizeof(double)), "zh_hist_distance");
+  const int32_t *ia = nullptr, *ib = nullptr;
+  if (!all) {
+    ZH_CU(c->d_ids.ensure((size_t)std::max<int64_t>(n, 1) * 2 * sizeof(int32_t)), "zh_hist_distance");
+    if (n > 0) {
+      ZH_CU(cudaMemcpyAsync(c->d_ids.p, a_ids, (size_t)n * 4, cudaMemcpyHostToDevice, c->stream), "zh_hist_distance");
+      ZH_CU(cudaMemcpyAsync(c->d_ids.as<int32_t>() + n, b_ids, (size_t)n * 4, cudaMemcpyHostToDevice, c->stream),
+            "zh_hist_distance");
+    }
+    ia = c->d_ids.as<int32_t>();
+    ib = ia + n;
+  }
+  ZH_CU(zh::launch_hist_distance(*c, kind, c->d_stats.as<int64_t>(), narrow, ia, ib, all ? 0 : n,
+                                 c->d_dist.as<double>()),
+        "zh_hist_distance");
+  if (n_out > 0)
+    ZH_CU(cudaMemcpyAsync(host_out, c->d_dist.p, (size_t)n_out * sizeof(double), cudaMemcpyDeviceToHost, c->stream),
+          "zh_hist_distance (D2H)");
+  ZH_CU(cudaStreamSynchronize(c->stream), "zh_hist_distance");
   return ZH_OK;
 }
 

@@ -72,6 +72,7 @@ struct Ctx {
   DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,
       d_pip, d_pip_cur, d_fcounts, d_pbits, d_remap, d_pip_grp, d_mixed_pk;
   DBuf d_stats;  // zonal statistics [P][8] (k_stats.cu)
+  DBuf d_summary, d_cdf, d_dist, d_ids;  // zonal summary [P][6], row CDFs, distances, pair ids (k_features.cu)
   int64_t n_cand = 0, n_bands = 0, n_band_entries = 0, n_inside = 0, n_isect = 0;
   // step 1 product and output
   DBuf d_tile_hist;
@@ -113,6 +114,9 @@ cudaError_t launch_touch(Ctx& c, const int32_t* remap, cudaStream_t s);  // k_to
 cudaError_t launch_fused(Ctx& c);  // steps 1 + 3 + 4 fused (k_fused.cu)
 cudaError_t launch_need_tiles(Ctx& c);  // d_need[t] = tile t has a pair (k_fused.cu)
 cudaError_t launch_zonal_stats(Ctx& c, int64_t* dstats);  // k_stats.cu
+cudaError_t launch_zonal_summary(Ctx& c, const int64_t* dstats, double* dout);  // k_features.cu
+cudaError_t launch_hist_distance(Ctx& c, int kind, const int64_t* dstats, bool narrow, const int32_t* ia,
+                                 const int32_t* ib, int64_t n, double* dout);  // k_features.cu
 cudaError_t launch_row_cost(Ctx& c, double* d_row_cost);  // k_fused.cu (shard planning)
 
 size_t device_bytes(const Ctx& c);

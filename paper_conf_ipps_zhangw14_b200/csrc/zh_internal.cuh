@@ -154,14 +154,18 @@ __host__ __device__ inline FastBins make_fast_bins(const BinP& b) {
   f.C2 = pk(C);
   f.nod2 = pk(b.nodata);
   f.use_nodata = b.use_nodata ? 1u : 0u;
-  // biased form: valid when nodata < L and the nodata index stays above the dummy slots
+  // biased form: valid when nodata < L, the nodata index stays above the dummy slots, and no value
+  // lies below nodata that would have to be counted: v - (nodata+1) wraps for v < nodata, which
+  // sends those cells to the dummy slots.  That is right in drop mode (v < nodata < lo is dropped)
+  // and vacuous for nodata = -32768; in clamp mode with a higher nodata they belong in bin 0.
   const int N1 = b.nodata + 1;
   f.Hb2 = pk(H);
   f.Nb2 = pk(N1);
   f.Lb2 = pk(L - N1);
   f.Cb2 = pk(C - N1);
   const int nod_idx = 0xFFFF - ((C - N1) & 0xFFFF);  // where a nodata cell lands
-  f.bias = (b.use_nodata && b.nodata < L && nod_idx >= hist_dummy(b.nbins) + 32) ? 1u : 0u;
+  f.bias = (b.use_nodata && b.nodata < L && (b.drop || b.nodata == -32768) && nod_idx >= hist_dummy(b.nbins) + 32)
+               ? 1u : 0u;
   return f;
 }
 

@@ -19,6 +19,10 @@ from . import _build
 # ZH_LIBZH: load another build of libzh (A/B experiments); default is the in-tree build.
 _LIB_PATH = os.environ.get("ZH_LIBZH", _build.LIB)
 
+ZH_DIST_L1, ZH_DIST_EMD, ZH_DIST_CHI2 = 0, 1, 2
+_DIST_KINDS = {"l1": ZH_DIST_L1, "emd": ZH_DIST_EMD, "chi2": ZH_DIST_CHI2}
+SUMMARY_FIELDS = ("count", "min", "max", "median", "mean", "std")
+
 ZH_OK, ZH_ERR_INVALID_ARG, ZH_ERR_UNSUPPORTED, ZH_ERR_OOM, ZH_ERR_CUDA, ZH_ERR_OVERFLOW, ZH_ERR_STATE = range(7)
 _STATUS = {0: "ZH_OK", 1: "ZH_ERR_INVALID_ARG", 2: "ZH_ERR_UNSUPPORTED", 3: "ZH_ERR_OOM", 4: "ZH_ERR_CUDA",
            5: "ZH_ERR_OVERFLOW", 6: "ZH_ERR_STATE"}
@@ -62,7 +66,7 @@ class zh_stats(ctypes.Structure):
 
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",
-           "zh_fused_update", "zh_zonal_stats", "zh_plan_rows",
+           "zh_fused_update", "zh_zonal_stats", "zh_zonal_summary", "zh_hist_distance", "zh_plan_rows",
            "zh_run", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
            "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy",
            "zh_trim_cache", "zh_cache_bytes"]
@@ -85,6 +89,8 @@ def _load():
         "zh_pip_update": (st, [vp]),
         "zh_fused_update": (st, [vp]),
         "zh_zonal_stats": (st, [vp, vp, vp]),
+        "zh_zonal_summary": (st, [vp, vp, vp]),
+        "zh_hist_distance": (st, [vp, i32, vp, vp, i64, vp]),
         "zh_plan_rows": (st, [ctypes.POINTER(zh_raster), ctypes.POINTER(zh_polygons), ctypes.POINTER(zh_options), i32,
                               vp, vp]),
         "zh_run": (st, [vp, vp]),
@@ -267,21 +273,33 @@ class ZonalHistogram:
         _check(LIB.zh_zonal_stats(self.h, out.ctypes.data if self.n_poly else None, None))
         return out
 
-    def zonal_stats(self, lo: int = 0, width: int = 1) -> dict:
-        """count, min, max, median, mean, std per polygon in value units (value of bin b =
-        lo + b * width), derived from zh_zonal_stats' exact integers."""
-        raw = self.zh_zonal_stats()
-        n = raw[:, 0].astype(np.float64)
-        s = raw[:, 4].astype(np.float64)
-        sq = raw[:, 5].view(np.uint64).astype(np.float64) + raw[:, 6].astype(np.float64) * 2.0 ** 64
-        with np.errstate(invalid="ignore", divide="ignore"):
-            mean_b = s / n
-            var_b = np.maximum(sq / n - mean_b * mean_b, 0.0)
-        empty = raw[:, 0] == 0
-        val = lambda b: np.where(empty, np.nan, lo + b * width)
-        return {"count": raw[:, 0], "min": val(raw[:, 1]), "max": val(raw[:, 2]), "median": val(raw[:, 3]),
-                "mean": np.where(empty, np.nan, lo + mean_b * width),
-                "std": np.where(empty, np.nan, np.sqrt(var_b) * width), "nonzero_bins": raw[:, 7]}
+    def zh_zonal_summary(self) -> np.ndarray:
+        """[n_poly, 6] float64: count, min, max, median, mean, std in value units, computed by libzh
+        from the exact integer statistics (zh.h states the rounding of each field)."""
+        out = np.zeros((self.n_poly, len(SUMMARY_FIELDS)), dtype=np.float64)
+        _check(LIB.zh_zonal_summary(self.h, out.ctypes.data if self.n_poly else None, None))
+        return out
+
+    def zonal_stats(self) -> dict:
+        """zh_zonal_summary as a dict of columns (value units of this context's bin mapping)."""
+        out = self.zh_zonal_summary()
+        return {f: out[:, i] for i, f in enumerate(SUMMARY_FIELDS)}
+
+    def zh_hist_distance(self, kind: str = "l1", a=None, b=None) -> np.ndarray:
+        """Distances between normalised polygon histograms (zh.h: l1, emd, chi2).  a, b: polygon id
+        sequences (pairwise, same length) -> [n]; both None -> the all-pairs [n_poly, n_poly] matrix."""
+        k = _DIST_KINDS[kind]
+        if a is None and b is None:
+            out = np.empty((self.n_poly, self.n_poly), dtype=np.float64)
+            _check(LIB.zh_hist_distance(self.h, k, None, None, 0, out.ctypes.data))
+            return out
+        ia = np.ascontiguousarray(a, dtype=np.int32)
+        ib = np.ascontiguousarray(b, dtype=np.int32)
+        if ia.shape != ib.shape or ia.ndim != 1:
+            raise ValueError("a and b must be 1-D sequences of the same length")
+        out = np.empty(ia.shape[0], dtype=np.float64)
+        _check(LIB.zh_hist_distance(self.h, k, ia.ctypes.data, ib.ctypes.data, ia.shape[0], out.ctypes.data))
+        return out
 
     def output_device(self):
         """The output as a torch CUDA tensor view (int64 for u64, int32 for u32 — same bits)."""

@@ -33,7 +33,7 @@ def test_library_exports_every_declared_symbol():
     assert not missing, missing
     from paper_conf_ipps_zhangw14_b200 import zh
     assert set(zh.EXPORTS) == set(_declared())
-    assert zh.LIB.zh_abi_version() == 5
+    assert zh.LIB.zh_abi_version() == 6
 
 
 def test_library_is_sm100a_sass():
@@ -115,6 +115,10 @@ def _mk(lib_zh, **over):
 @pytest.mark.parametrize("over,status", [
     ({"o__tile": 0}, 1), ({"b__nbins": 0}, 1), ({"b__width": 0}, 1), ({"r__pitch": 8}, 1),
     ({"r__row0": 3, "r__nrows": 8}, 1), ({"r__nrows": 20}, 1), ({"b__nbins": 1 << 20}, 1),
+    # nodata must be an int16 value (a wider one would alias a real value in the packed bin path)
+    ({"b__use_nodata": 1, "b__nodata": 65535}, 1), ({"b__use_nodata": 1, "b__nodata": -32769}, 1),
+    # uint32 shared histograms: T^2 < 2^31
+    ({"o__tile": 46341}, 2),
 ])
 def test_create_rejects_malformed_input(over, status):
     from paper_conf_ipps_zhangw14_b200 import zh

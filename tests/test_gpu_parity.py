@@ -156,7 +156,12 @@ def test_flipped_geotransforms(tiny, cuda_device, flip):
 
 
 @pytest.mark.parametrize("lo,width,nbins,drop,nodata", [(0, 1, 256, True, -32768), (-100, 3, 77, False, None),
-                                                         (20, 7, 9, True, -32768), (-20, 1, 300, False, 150)])
+                                                         (20, 7, 9, True, -32768), (-20, 1, 300, False, 150),
+                                                         # nodata below lo with values below nodata
+                                                         # (tiny: -157..401): clamp counts them in
+                                                         # bin 0, drop drops them
+                                                         (0, 1, 256, False, -100), (0, 1, 256, True, -100),
+                                                         (-50, 1, 5000, False, -120), (-150, 1, 600, False, -151)])
 def test_bin_mappings(tiny, cuda_device, lo, width, nbins, drop, nodata):
     cfg, P, R, _ = tiny
     H = oracle.o1(R, cfg.gt, P, oracle.make_bins(nbins, lo=lo, width=width, nodata=nodata, oor_drop=drop))
@@ -318,10 +323,10 @@ def test_zonal_stats_match_oracle(tiny, cuda_device, out_u64):
                                    out_u64=out_u64, fused=fused) as z:
                 z.run()
                 got = z.zh_zonal_stats()
-                derived = z.zonal_stats(lo=lo)
+                derived = z.zonal_stats()
             assert (got == want).all()
             nz = want[:, 0] > 0
-            assert np.allclose(derived["min"][nz], lo + want[nz, 1])
+            assert (derived["min"][nz] == lo + want[nz, 1]).all()
             assert (derived["count"] == want[:, 0]).all()
 
 
@@ -350,3 +355,45 @@ def test_large_and_generic_histograms(tiny, cuda_device, nbins, lo, width):
     t = device_raster(cfg.dem, cfg.rows, cfg.cols)
     G = gpu_hist(t, cfg.gt, P, nbins, 128, cfg.cols, lo=lo, width=width, nodata=cfg.nodata)
     assert (G == H).all()
+
+
+def test_lonlat_vertices_exactly_on_centres(cuda_device):
+    """Non-dyadic equality cases: a 1-arc-second lon/lat geotransform with polygon
+    vertices placed EXACTLY on computed cell centres — x = gt0 + (c + 0.5) gt1, y = gt3 + (r + 0.5) gt5,
+    the same binary64 expressions both sides evaluate — so centre rows meet vertices (ya == yc: the
+    half-open straddle rule at its boundary, k_edges' exact row intervals), vertical edges sit on
+    centre columns (xi == xc: not a crossing) and shared borders pass through centres.  GPU ==
+    literal O0 (no prefilter) at several tile sizes, both paths."""
+    ARC = 1.0 / 3600.0
+    rows, cols = 600, 704
+    gt = (-100.0, ARC, 0.0, 40.0, 0.0, -ARC)
+    xc = lambda c: gt[0] + (c + 0.5) * gt[1]
+    yc = lambda r: gt[3] + (r + 0.5) * gt[5]
+    rng = np.random.default_rng(31)
+    polys = []
+    for _ in range(14):  # star-shaped, vertices on centres
+        cr, cc = rng.integers(60, rows - 60), rng.integers(60, cols - 60)
+        n = int(rng.integers(5, 40))
+        th = np.sort(rng.uniform(0, 2 * np.pi, n))
+        rad = rng.uniform(8, 55, n)
+        r = np.clip(np.rint(cr + rad * np.sin(th)), 0, rows - 1).astype(int)
+        c = np.clip(np.rint(cc + rad * np.cos(th)), 0, cols - 1).astype(int)
+        polys.append([(np.array([xc(v) for v in c]), np.array([yc(v) for v in r]))])
+    for _ in range(6):  # axis-aligned boxes with corners on centres, one with a hole on centres
+        r0, c0 = rng.integers(0, rows - 80), rng.integers(0, cols - 80)
+        h, w = rng.integers(5, 79, 2)
+        box = (np.array([xc(c0), xc(c0 + w), xc(c0 + w), xc(c0)]), np.array([yc(r0), yc(r0), yc(r0 + h), yc(r0 + h)]))
+        polys.append([box])
+    r0, c0 = 200, 300
+    outer = (np.array([xc(c0), xc(c0 + 90), xc(c0 + 90), xc(c0)]), np.array([yc(r0), yc(r0), yc(r0 + 70), yc(r0 + 70)]))
+    hole = (np.array([xc(c0 + 10), xc(c0 + 30), xc(c0 + 30), xc(c0 + 10)]),
+            np.array([yc(r0 + 10), yc(r0 + 10), yc(r0 + 50), yc(r0 + 50)]))
+    polys.append([outer, hole])
+    P = from_rings(polys)
+    spec = TINY.dem
+    R = fill_host(spec, cols, 0, 0, rows, cols)
+    H = oracle.o0(R, gt, P, oracle.make_bins(256, nodata=-32768))
+    assert H.sum() > 0
+    t = device_raster(spec, rows, cols)
+    for tile in (16, 64, 100, 128, 704):
+        assert (gpu_hist(t, gt, P, 256, tile, cols, nodata=-32768) == H).all(), tile

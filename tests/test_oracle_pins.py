@@ -272,3 +272,24 @@ def test_representative_point_offsets():
         assert [int(v) for v in fn(R, gt, P, bins)[:, 0]] == [28, 28]
     # centre == explicit (0.5, 0.5)
     assert (oracle.o1(R, gt, P, bins, rep=(0.5, 0.5)) == oracle.o1(R, gt, P, bins)).all()
+
+
+def test_centre_operation_order_non_dyadic():
+    """R7: the centre is gt0 + ((c + 0.5) * gt1), three binary64 ops in that order (the reading both
+    sides implement).  Under a lon/lat geotransform (1 arc-second, not dyadic) other orders give
+    other doubles, so this pins the oracle's order: numpy float64 scalars (IEEE, no FMA) evaluate
+    the stated order, and the alternative orders must disagree on some cells (the check bites)."""
+    from synth.configs import CONUS
+    gt = CONUS.gt
+    rng = np.random.default_rng(7)
+    rr = rng.integers(0, CONUS.rows, 2000)
+    cc = rng.integers(0, CONUS.cols, 2000)
+    alt_x = alt_y = 0
+    for r, c in zip(rr, cc):
+        xc, yc = oracle.centre(gt, int(r), int(c))
+        want_x = np.float64(gt[0]) + (np.float64(c) + np.float64(0.5)) * np.float64(gt[1])
+        want_y = np.float64(gt[3]) + (np.float64(r) + np.float64(0.5)) * np.float64(gt[5])
+        assert xc == want_x and yc == want_y
+        alt_x += (np.float64(gt[0]) + np.float64(c) * np.float64(gt[1]) + np.float64(0.5) * np.float64(gt[1])) != xc
+        alt_y += (np.float64(gt[3]) + np.float64(r) * np.float64(gt[5]) + np.float64(0.5) * np.float64(gt[5])) != yc
+    assert alt_x > 0 and alt_y > 0
