@@ -229,15 +229,16 @@ zh_status zh_zonal_summary(zh_ctx ctx, double* host_out, double** dptr);
  * as feature vectors for ... computing various distance measurements which can be used for
  * subsequent clustering").  Between the NORMALISED histograms p = H_a / n_a, q = H_b / n_b of
  * polygons a and b (n = count):
- *   ZH_DIST_L1   sum_b |p_b - q_b|                       = RN(RN(RN(N) / n_a) / n_b),
+ *   ZH_DIST_L1   sum_b |p_b - q_b|                       = RN(RN(RN(N) / n_1) / n_2),
  *                N = sum_b |H_a[b]*n_b - H_b[b]*n_a|  (an exact 128-bit integer: bit-exact)
  *   ZH_DIST_EMD  sum_b |P_b - Q_b|, P, Q the cumulative distributions (1-D earth mover's
  *                distance in bin units; times width for value units); same form with the
  *                cumulative counts C_a[b] = sum_{b' <= b} H_a[b'] in place of H (bit-exact)
  *   ZH_DIST_CHI2 1/2 sum_{b: p_b + q_b > 0} (p_b - q_b)^2 / (p_b + q_b), evaluated as
- *                0.5 * RN(RN(sum_b RN(RN(d^2) / s)) / n_a) / n_b) with d = RN(|H_a[b] n_b - H_b[b] n_a|),
+ *                0.5 * RN(RN(sum_b RN(RN(d^2) / s)) / n_1) / n_2) with d = RN(|H_a[b] n_b - H_b[b] n_a|),
  *                s = RN(H_a[b] n_b + H_b[b] n_a), the sum in an unspecified order: relative
  *                error <= (nbins + 8) * 2^-53
+ * (n_1 = min(n_a, n_b), n_2 = max(n_a, n_b): the result is symmetric in a and b.)
  * NaN when either polygon is empty.  a_ids, b_ids: HOST int32 arrays of n polygon ids (each in
  * [0, n_poly), else INVALID_ARG); host_out[i] = d(a_ids[i], b_ids[i]).  a_ids = b_ids = NULL:
  * ALL pairs, host_out is [n_poly][n_poly] row-major (n ignored), symmetric, zero diagonal for

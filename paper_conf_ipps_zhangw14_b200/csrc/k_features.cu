@@ -178,9 +178,10 @@ struct PairAcc {
 template <int kKind>
 __device__ __forceinline__ double finish(const U128& n, double c, unsigned long long na, unsigned long long nb) {
   if (na == 0 || nb == 0) return __longlong_as_double(0x7ff8000000000000ll);
-  const double da = __ull2double_rn(na), db = __ull2double_rn(nb);
-  if (kKind == ZH_DIST_CHI2) return 0.5 * __ddiv_rn(__ddiv_rn(c, da), db);
-  return __ddiv_rn(__ddiv_rn(u128_to_double_rn(n), da), db);
+  // divide by the smaller count first: the rounding is then symmetric in (a, b)
+  const double d1 = __ull2double_rn(na < nb ? na : nb), d2 = __ull2double_rn(na < nb ? nb : na);
+  if (kKind == ZH_DIST_CHI2) return 0.5 * __ddiv_rn(__ddiv_rn(c, d1), d2);
+  return __ddiv_rn(__ddiv_rn(u128_to_double_rn(n), d1), d2);
 }
 
 // List mode: one warp per (a, b) pair, lanes over bins; partial sums combined in a fixed order.

@@ -89,7 +89,12 @@ def test_hist_distances(tiny_gpu, cuda_device, monkeypatch, kind, wide):
         L = z.zh_hist_distance(kind, a, b)
         M = z.zh_hist_distance(kind)
         few = z.zh_hist_distance(kind, [3], [3])
-    assert np.array_equal(L.reshape(P.n_poly, P.n_poly), M, equal_nan=True)
+    L = L.reshape(P.n_poly, P.n_poly)
+    if kind == "chi2":  # the two modes sum the bins in different orders
+        assert np.allclose(L, M, rtol=(cfg.nbins + 8) * 2 * U, atol=0, equal_nan=True)
+    else:
+        assert np.array_equal(L, M, equal_nan=True)
+    assert np.array_equal(M, M.T, equal_nan=True)
     n = H.sum(axis=1).astype(object)
     for i, j in zip(a, b):
         e = F.distance_exact(H, kind, int(i), int(j))
@@ -102,7 +107,8 @@ def test_hist_distances(tiny_gpu, cuda_device, monkeypatch, kind, wide):
         else:
             N = e * n[i] * n[j]
             assert N.denominator == 1
-            assert g == float(N.numerator) / float(n[i]) / float(n[j]), (i, j)  # bit-exact
+            n1, n2 = sorted((int(n[i]), int(n[j])))
+            assert g == float(N.numerator) / float(n1) / float(n2), (i, j)  # bit-exact
             assert abs(Fraction(g) - e) <= 3 * U * e
     assert few[0] == 0.0 and (np.diag(M)[n > 0] == 0).all()
 

@@ -108,7 +108,8 @@ def _features(t, cfg, P, H):
                 assert abs(Fraction(g[i]) - e) <= (cfg.nbins + 8) * U * e
             else:
                 N = e * int(n[x]) * int(n[y])
-                assert g[i] == float(N.numerator) / float(int(n[x])) / float(int(n[y]))
+                n1, n2 = sorted((int(n[x]), int(n[y])))
+                assert g[i] == float(N.numerator) / float(n1) / float(n2)
 
 
 def test_state_full_size(cuda_device):
