@@ -23,13 +23,6 @@
 #define ZH_PURE_MINB 3  // CTAs of 512 threads per SM the pure-tile kernel is compiled for (register cap)
 #endif
 
-#ifndef ZH_EXACT_GRID
-#define ZH_EXACT_GRID 1  // 1: step-4 grids sized from the list counts (host reads them during k_fused_pure)
-#endif
-
-#ifndef ZH_PAR_SIDE
-#define ZH_PAR_SIDE 0  // 1: k_parity on the side stream, beside k_fused_pure (measured slower: registers)
-#endif
 
 namespace zh {
 
@@ -421,36 +414,22 @@ cudaError_t launch_fused(Ctx& c) {
   // mixed tiles, split form: the parity bitmaps of every cell-in-polygon pair are built on the side
   // stream WHILE the pure-tile kernel streams the pure tiles (FP64-latency work beside HBM-bound
   // work), then the cell kernel runs once both are done
-  const bool split = c.pip_split != 0 || c.cover != 0;
-  // exact grids for the step-4 kernels: the list sizes are copied to the host behind the list
-  // kernels and read while the pure-tile kernel runs (no CTAs that only find they have no work)
-  const bool exact = split && ZH_EXACT_GRID;
-  int64_t n_pip = NI + NX, n_grp = NI + NX;
-  if (split) {
-    if ((e = pip_prepare(c, NI + NX)) != cudaSuccess) return e;
-  }
-  if (exact) {
-    cudaMemcpyAsync(c.pinned_counts + 8, c.d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c.stream);
-    cudaEventRecord(c.ev_counts, c.stream);
-  }
+  // exact grid for the cell kernel: the list sizes are copied to the host behind the list kernels
+  // and read while the pure-tile kernel runs (no CTAs that only find they have no work)
+  if ((e = pip_prepare(c, NI + NX)) != cudaSuccess) return e;
+  cudaMemcpyAsync(c.pinned_counts + 8, c.d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c.stream);
+  cudaEventRecord(c.ev_counts, c.stream);
   auto parity = [&](int64_t grid) -> cudaError_t {
     cudaError_t pe;
-    if (c.timing) cudaEventRecord(c.ev[13], ZH_PAR_SIDE ? c.side : c.stream);
-    if ((pe = launch_parity(c, c.d_pip.as<int2>(), grid, c.d_fcounts.as<int64_t>() + 1,
-                            ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess)
+    if (c.timing) cudaEventRecord(c.ev[13], c.stream);
+    if ((pe = launch_parity(c, c.d_pip.as<int2>(), grid, c.d_fcounts.as<int64_t>() + 1, c.stream)) != cudaSuccess)
       return pe;
     if (c.cover) {  // R15: cells an edge reaches join the parity bits (k_touch.cu)
-      if ((pe = launch_touch(c, c.d_remap.as<int32_t>(), ZH_PAR_SIDE ? c.side : c.stream)) != cudaSuccess) return pe;
+      if ((pe = launch_touch(c, c.d_remap.as<int32_t>(), c.stream)) != cudaSuccess) return pe;
     }
-    if (c.timing) cudaEventRecord(c.ev[14], ZH_PAR_SIDE ? c.side : c.stream);
+    if (c.timing) cudaEventRecord(c.ev[14], c.stream);
     return cudaSuccess;
   };
-  if (split && !exact) {
-    cudaEventRecord(c.ev_fork, c.stream);
-    cudaStreamWaitEvent(c.side, c.ev_fork, 0);
-    if ((e = parity(NI + NX)) != cudaSuccess) return e;
-    cudaEventRecord(c.ev_join, c.side);
-  }
   // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
   if (c.timing) cudaEventRecord(c.ev[10], c.stream);
   if (NI > 0) {
@@ -478,35 +457,22 @@ cudaError_t launch_fused(Ctx& c) {
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
   if (c.timing) cudaEventRecord(c.ev[11], c.stream);
-  if (split) {
-    if (exact) {
-      if ((e = cudaEventSynchronize(c.ev_counts)) != cudaSuccess) return e;
-      n_pip = c.pinned_counts[8 + 1];
-      n_grp = c.pinned_counts[8 + 4];
-      if (n_pip > 0) {
-        if ((e = parity(n_pip)) != cudaSuccess) return e;
-      } else if (c.timing) {
-        cudaEventRecord(c.ev[13], c.stream);
-        cudaEventRecord(c.ev[14], c.stream);
-      }
-    } else {
-      cudaStreamWaitEvent(c.stream, c.ev_join, 0);
-    }
-    if (c.timing) cudaEventRecord(c.ev[15], c.stream);
-    if (grouped)
-      e = n_grp > 0 ? launch_mixed_cells(c, c.d_pip.as<int2>(), c.d_pip_grp.as<int2>(), n_grp,
-                                         c.d_fcounts.as<int64_t>() + 4)
-                    : cudaSuccess;
-    else
-      e = n_pip > 0 ? launch_pip_cells(c, c.d_pip.as<int2>(), n_pip, c.d_fcounts.as<int64_t>() + 1) : cudaSuccess;
-  } else {
-    if (c.timing) {
-      cudaEventRecord(c.ev[13], c.stream);
-      cudaEventRecord(c.ev[14], c.stream);
-      cudaEventRecord(c.ev[15], c.stream);
-    }
-    e = launch_pip_list(c, c.d_pip.as<int2>(), NI + NX, c.d_fcounts.as<int64_t>() + 1);
+  if ((e = cudaEventSynchronize(c.ev_counts)) != cudaSuccess) return e;
+  const int64_t n_pip = c.pinned_counts[8 + 1];
+  const int64_t n_grp = c.pinned_counts[8 + 4];
+  if (n_pip > 0) {
+    if ((e = parity(n_pip)) != cudaSuccess) return e;
+  } else if (c.timing) {
+    cudaEventRecord(c.ev[13], c.stream);
+    cudaEventRecord(c.ev[14], c.stream);
   }
+  if (c.timing) cudaEventRecord(c.ev[15], c.stream);
+  if (grouped)
+    e = n_grp > 0 ? launch_mixed_cells(c, c.d_pip.as<int2>(), c.d_pip_grp.as<int2>(), n_grp,
+                                       c.d_fcounts.as<int64_t>() + 4)
+                  : cudaSuccess;
+  else
+    e = n_pip > 0 ? launch_pip_cells(c, c.d_pip.as<int2>(), n_pip, c.d_fcounts.as<int64_t>() + 1) : cudaSuccess;
   if (c.timing) cudaEventRecord(c.ev[12], c.stream);
   return e;
 }

@@ -158,7 +158,7 @@ __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ 
                                                     const int2* __restrict__ erows, const int4* __restrict__ mbb,
                                                     const int64_t* __restrict__ band_base, int T, int mode,
                                                     int32_t* __restrict__ band_cnt, const int32_t* __restrict__ band_off,
-                                                    int32_t* __restrict__ band_edges) {
+                                                    int32_t* __restrict__ band_edges, int32_t* __restrict__ band_poly) {
   __shared__ int32_t sc[kSmemBands];
   const int k = blockIdx.x;
   const int4 m = mbb[k];
@@ -167,6 +167,8 @@ __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ 
   const int64_t bb = band_base[k];
   const bool in_smem = nb <= kSmemBands;
   int32_t* cnt = in_smem ? sc : nullptr;
+  if (mode == 0)
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) band_poly[bb + i] = k;  // band -> polygon
   if (in_smem) {
     for (int i = threadIdx.x; i < nb; i += blockDim.x) sc[i] = mode == 0 ? 0 : band_off[bb + i];
     __syncthreads();
@@ -240,12 +242,13 @@ __global__ void __launch_bounds__(256) k_mark(const int32_t* __restrict__ pro, c
 __global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges, const int2* __restrict__ erows,
                                                   const int32_t* __restrict__ band_off,
                                                   const int32_t* __restrict__ band_edges,
-                                                  const int64_t* __restrict__ band_base, int P, Geo g, RasterP rp,
+                                                  const int64_t* __restrict__ band_base,
+                                                  const int32_t* __restrict__ band_poly, Geo g, RasterP rp,
                                                   const int4* __restrict__ mbb, const int64_t* __restrict__ cand_off,
                                                   uint8_t* __restrict__ cls, int dwords) {
   extern __shared__ uint32_t D[];
   const int64_t band = blockIdx.x;
-  const int k = (int)(upper_bound_i64(band_base, P + 1, band) - 1);
+  const int k = band_poly[band];
   const int4 m = mbb[k];
   const int tr = m.z + (int)(band - band_base[k]);
   const int wk = m.y - m.x + 1;
@@ -393,6 +396,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   if ((e = c.d_band_off.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
   if ((e = c.d_band_cur.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
   if ((e = c.d_band_edges.ensure(sizeof(int32_t) * (size_t)ne)) != cudaSuccess) return e;
+  if ((e = c.d_band_poly.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
   if ((e = c.d_class.ensure((size_t)nc)) != cudaSuccess) return e;
   if ((e = c.d_flags.ensure(sizeof(uint64_t) * (size_t)nc)) != cudaSuccess) return e;
   if ((e = c.d_flag_pos.ensure(sizeof(uint64_t) * (size_t)nc)) != cudaSuccess) return e;
@@ -401,7 +405,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   if (V > 0 && nb > 0) {
     k_poly_bands<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
                                           c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 0,
-                                          c.d_band_cnt.as<int32_t>(), nullptr, nullptr);
+                                          c.d_band_cnt.as<int32_t>(), nullptr, nullptr, c.d_band_poly.as<int32_t>());
     c.launches += 1;
   }
   if (nb > 0) {
@@ -412,7 +416,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
       k_poly_bands<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
                                             c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 1,
                                             c.d_band_cur.as<int32_t>(), c.d_band_off.as<int32_t>(),
-                                            c.d_band_edges.as<int32_t>());
+                                            c.d_band_edges.as<int32_t>(), nullptr);
       c.launches += 1;
     }
   }
@@ -431,7 +435,8 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
       const int dwords = c.rp.TC / 32 + 2;
       k_classify<<<(unsigned)nb, 128, sizeof(uint32_t) * dwords, c.stream>>>(
           c.d_edges.as<Edge>(), c.d_erows.as<int2>(), c.d_band_off.as<int32_t>(), c.d_band_edges.as<int32_t>(),
-          c.d_band_base.as<int64_t>(), P, c.geo, c.rp, c.d_mbb.as<int4>(), c.d_cand_off.as<int64_t>(),
+          c.d_band_base.as<int64_t>(), c.d_band_poly.as<int32_t>(), c.geo, c.rp, c.d_mbb.as<int4>(),
+          c.d_cand_off.as<int64_t>(),
           c.d_class.as<uint8_t>(), dwords);
       c.launches += 1;
     }

@@ -36,14 +36,6 @@ namespace zh {
 #endif
 constexpr int kPipThreads = ZH_PIP_THREADS;  // k_pip_cells
 
-template <int kMode, bool kU64, bool kRep>
-__global__ void __launch_bounds__(256, ZH_PIP_MINB) k_pip(PipP p) {
-  if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
-  extern __shared__ __align__(16) uint32_t sh[];
-  __shared__ LongQ lq;
-  pip_pair_body<kMode, kU64, kRep>(p, blockIdx.x, sh, &lq);
-}
-
 // Split form (zh_pip.cuh): parity bitmaps of every pair, then the cells.
 #ifndef ZH_PAR_THREADS
 #define ZH_PAR_THREADS 128
@@ -120,12 +112,6 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev) {
   p.bmo = 0;
   return p;
 }
-
-size_t pip_smem(const Ctx& c, const PipP& p) {
-  return (size_t)hist_words(c.bp.nbins) * 4 + (size_t)p.rc * p.wpr * 4;
-}
-
-static cudaError_t launch_pip_fused_body(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev);
 
 static int pip_mode(const Ctx& c) {
   const FastBins fb = make_fast_bins(c.bp);
@@ -230,39 +216,14 @@ cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64
   return cudaGetLastError();
 }
 
+// Four-step step 4 over step 2's intersecting pairs (bitmap slot = isect index).
 cudaError_t launch_pip_list(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
   if (grid == 0) return cudaSuccess;
-  if (c.pip_split || c.cover) {
-    cudaError_t e = pip_prepare(c, grid);
-    if (e != cudaSuccess) return e;
-    if ((e = launch_parity(c, pairs, grid, n_dev, c.stream)) != cudaSuccess) return e;
-    if (c.cover && pairs == c.d_isect.as<int2>() && (e = launch_touch(c, nullptr, c.stream)) != cudaSuccess) return e;
-    return launch_pip_cells(c, pairs, grid, n_dev);
-  }
-  return launch_pip_fused_body(c, pairs, grid, n_dev);
-}
-
-static cudaError_t launch_pip_fused_body(Ctx& c, const int2* pairs, int64_t grid, const int64_t* n_dev) {
-  if (grid == 0) return cudaSuccess;
-  PipP p = pip_params(c, pairs, n_dev);
-  const size_t smem = pip_smem(c, p);
-  void (*k)(PipP);
-  const int mode = fast_bins_ok(c.bp) ? (p.fb.bias ? 4 : (c.bp.use_nodata ? 3 : 2)) : (c.bp.width == 1 ? 0 : 1);
-  const bool rep = !(c.geo.ox == 0.5 && c.geo.oy == 0.5);
-#define ZH_PIP_K(M) (c.out_u64 ? (rep ? k_pip<M, true, true> : k_pip<M, true, false>) \
-                               : (rep ? k_pip<M, false, true> : k_pip<M, false, false>))
-  switch (mode) {
-    case 0: k = ZH_PIP_K(0); break;
-    case 1: k = ZH_PIP_K(1); break;
-    case 2: k = ZH_PIP_K(2); break;
-    case 3: k = ZH_PIP_K(3); break;
-    default: k = ZH_PIP_K(4); break;
-  }
-#undef ZH_PIP_K
-  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k<<<(unsigned)grid, 256, smem, c.stream>>>(p);
-  c.launches += 1;
-  return cudaGetLastError();
+  cudaError_t e = pip_prepare(c, grid);
+  if (e != cudaSuccess) return e;
+  if ((e = launch_parity(c, pairs, grid, n_dev, c.stream)) != cudaSuccess) return e;
+  if (c.cover && pairs == c.d_isect.as<int2>() && (e = launch_touch(c, nullptr, c.stream)) != cudaSuccess) return e;
+  return launch_pip_cells(c, pairs, grid, n_dev);
 }
 
 }  // namespace zh

@@ -11,9 +11,6 @@
 #ifndef ZH_PIP_GROUP_DEFAULT
 #define ZH_PIP_GROUP_DEFAULT 1
 #endif
-#ifndef ZH_PIP_SPLIT_DEFAULT
-#define ZH_PIP_SPLIT_DEFAULT 1
-#endif
 
 namespace zh {
 
@@ -59,7 +56,6 @@ struct Ctx {
   int32_t force_isect = 0;
   int32_t cover = 0;  // R15: closed cell rectangle meets the closed polygon (k_touch.cu)
   int32_t pip_group = ZH_PIP_GROUP_DEFAULT;  // fused path: mixed-tile groups of <= 2 pairs (k_mixed_cells) or one CTA per pair
-  int32_t pip_split = ZH_PIP_SPLIT_DEFAULT;  // step 4 as k_parity + k_pip_cells (1) or one k_pip kernel per pair (0)
   cudaStream_t stream = nullptr;
   // polygons (device)
   int32_t P = 0, R = 0, V = 0;
@@ -68,6 +64,7 @@ struct Ctx {
   DBuf d_edges, d_erows, d_mbb, d_ncand, d_nband, d_cand_off, d_band_base;
   DBuf d_band_cnt, d_band_off, d_band_cur, d_band_edges, d_class, d_flags, d_flag_pos;
   DBuf d_inside, d_isect, d_counts, d_cub;
+  DBuf d_band_poly;  // band -> polygon
   // fused path lists (k_fused.cu)
   DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,
       d_pip, d_pip_cur, d_fcounts, d_pbits, d_remap, d_pip_grp, d_mixed_pk;

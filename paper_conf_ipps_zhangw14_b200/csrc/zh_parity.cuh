@@ -121,20 +121,6 @@ __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, i
   __syncthreads();
 }
 
-// Step 2: in place, rows [0, ch) of bm become parity (inside) bits.  Thread per row.
-__device__ __forceinline__ void suffix_xor_rows(uint32_t* __restrict__ bm, int wpr, int ch) {
-  for (int lr = threadIdx.x; lr < ch; lr += blockDim.x) {
-    uint32_t* row = bm + lr * wpr;
-    uint32_t carry = 0;
-    for (int wi = wpr - 1; wi >= 0; --wi) {
-      uint32_t t = row[wi];
-      t ^= t >> 1; t ^= t >> 2; t ^= t >> 4; t ^= t >> 8; t ^= t >> 16;
-      row[wi] = (t >> 1) ^ (carry ? 0xFFFFFFFFu : 0u);
-      carry ^= (t & 1u);
-    }
-  }
-}
-
 // Step 2 for the split form: rows [0, ch) of bm become parity bits written straight to `out`
 // (row stride wpo = ceil(w / 32) words, the word wpr - 1 = wpo only carries the "all cells" flips).
 // Thread per row; with wpo % 4 == 0 the row is produced 4 words at a time and stored as 16 bytes.

@@ -1,4 +1,4 @@
-// zh_pip.cuh — step 4 for one (tile, polygon) pair, shared by k_pip and the fused kernel.
+// zh_pip.cuh — step 4 device code: the per-pair parity form (A/B reference) and the cell passes.
 #pragma once
 #include <type_traits>
 
@@ -42,128 +42,6 @@ struct PipP {
 
 struct Ctx;  // zh_ctx.h
 PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev);  // k_pip.cu
-size_t pip_smem(const Ctx& c, const PipP& p);
-
-// One (tile, polygon) pair: parity bitmap, masked cell pass, flush (the whole step-4 work of a pair).
-// `sh` holds hist_words(nbins) + rc * wpr words; `lq` must hold n = 0 (published by a barrier before
-// the first crossing phase — the body's first barrier does that).
-// kMode as in k_tile_hist: 0/1 generic (w1 / w>1), 2 + kForm packed.
-template <int kMode, bool kU64, bool kRep>
-__device__ __forceinline__ void pip_pair_body(const PipP& p, int64_t pair_idx, uint32_t* __restrict__ sh,
-                                              LongQ* lqp) {
-  LongQ& lq = *lqp;
-  const int HW = hist_words(p.bp.nbins);
-  uint32_t* hist = sh;
-  uint32_t* bm = sh + HW;
-  if (threadIdx.x == 0) lq.n = 0;
-  const RasterP& rp = p.rp;
-  const Geo& g = p.g;
-
-  const int2 pr = p.isect[pair_idx];
-  const int tile = pr.x, k = pr.y;
-  const TileGeom t = tile_geom<kRep>(rp, g, tile);
-  const int64_t r0 = t.r0, c0 = t.c0;
-  const int h = t.h, w = t.w;
-  const int4 m = p.mbb[k];
-  const int64_t band = p.band_base[k] + ((int)(r0 / rp.T) - m.z);
-  const int e0 = p.band_off[band], e1 = p.band_off[band + 1];
-
-  for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
-    *reinterpret_cast<uint4*>(&hist[i]) = make_uint4(0, 0, 0, 0);
-  const uint32_t dummy = (uint32_t)hist_dummy(p.bp.nbins) + (threadIdx.x & 31);
-  const uint32_t dum2 = dummy * 0x10001u;
-
-  const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
-  const int nk = (int)(k1 - k0);
-  const int64_t pitch = rp.pitch;
-  const FastBins fb = p.fb;
-
-  for (int cr = 0; cr < h; cr += p.rc) {
-    const int ch = min(p.rc, h - cr);
-    const int64_t rlo = r0 + cr, rhi = rlo + ch;  // global rows of this chunk
-    for (int i = threadIdx.x; i < ch * p.wpr; i += blockDim.x) bm[i] = 0;
-    __syncthreads();
-    crossings_to_bitmap<kRep>(bm, p.wpr, e0, e1, p.band_edges, p.edges, p.erows, g, t, rlo, rhi, &lq);
-    suffix_xor_rows(bm, p.wpr, ch);
-    __syncthreads();
-    // ---- cells: stream the chunk's rows, count inside cells (fully-outside vectors are not read)
-    const int16_t* base = rp.data + (rlo - rp.row0) * pitch + k0 * 8;
-    if (nk <= (int)blockDim.x) {
-      const int rpi = blockDim.x / nk;
-      const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
-      // kA: the tile starts on a vector boundary (c0 % 8 == 0, e.g. T % 8 == 0), so each thread's 8
-      // parity bits are one byte of one bitmap word (no straddling)
-      auto run = [&](auto aligned) {
-        constexpr bool kA = decltype(aligned)::value;
-        const int64_t cs = (k0 + kk) * 8;
-        const uint32_t cskip = cols_skip8(cs, c0, w);
-        const int lc0 = (int)(cs - c0);
-        const int wi = lc0 >> 5, bsh = lc0 & 31;
-        auto pbits = [&](int lr) -> uint32_t {
-          if (kA) return (bm[lr * p.wpr + wi] >> bsh) & 0xFFu;
-          return bits8(bm + lr * p.wpr, p.wpr, lc0);
-        };
-        const int16_t* ptr = base + (int64_t)rs * pitch + kk * 8;
-        const int64_t step = (int64_t)rpi * pitch;
-        int lr = rs;
-        // two rows per iteration: both skip masks first, then both loads in flight
-        for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
-          const uint32_t s0 = cskip | (~pbits(lr) & 0xFFu);
-          const uint32_t s1 = cskip | (~pbits(lr + rpi) & 0xFFu);
-          uint4 q0 = make_uint4(0, 0, 0, 0), q1 = make_uint4(0, 0, 0, 0);
-          if (s0 != 0xFFu) q0 = ld_stream16(ptr);
-          if (s1 != 0xFFu) q1 = ld_stream16(ptr + step);
-          if (s0 != 0xFFu) {
-            if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q0, s0, fb, dum2);
-            else count8_generic<kMode == 0>(hist, q0, s0, p.bp, dummy);
-          }
-          if (s1 != 0xFFu) {
-            if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q1, s1, fb, dum2);
-            else count8_generic<kMode == 0>(hist, q1, s1, p.bp, dummy);
-          }
-        }
-        for (; lr < ch; lr += rpi, ptr += step) {
-          const uint32_t skip = cskip | (~pbits(lr) & 0xFFu);
-          if (skip == 0xFFu) continue;
-          const uint4 q = ld_stream16(ptr);
-          if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q, skip, fb, dum2);
-          else count8_generic<kMode == 0>(hist, q, skip, p.bp, dummy);
-        }
-      };
-      if (rs < rpi) {
-        if ((c0 & 7) == 0) run(std::integral_constant<bool, true>{});
-        else run(std::integral_constant<bool, false>{});
-      }
-    } else {
-      for (int lr = 0; lr < ch; ++lr) {
-        for (int kk = threadIdx.x; kk < nk; kk += blockDim.x) {
-          const int64_t cs = (k0 + kk) * 8;
-          const uint32_t skip = cols_skip8(cs, c0, w) | (~bits8(bm + lr * p.wpr, p.wpr, (int)(cs - c0)) & 0xFFu);
-          if (skip == 0xFFu) continue;
-          const uint4 q = ld_stream16(base + (int64_t)lr * pitch + kk * 8);
-          if (kMode >= 2) count8_fast<kMode - 2, true>(hist, q, skip, fb, dum2);
-          else count8_generic<kMode == 0>(hist, q, skip, p.bp, dummy);
-        }
-      }
-    }
-    __syncthreads();
-  }
-  // ---- flush the pair's histogram
-  const int nbins = p.bp.nbins;
-  const int64_t orow = (int64_t)k * nbins;
-  for (int b = threadIdx.x * 4; b < nbins; b += blockDim.x * 4) {  // 16-byte reads, zero vectors skipped
-    const uint4 v = *reinterpret_cast<const uint4*>(&hist[kOff + b]);
-    if (!(v.x | v.y | v.z | v.w)) continue;
-    const uint32_t vs[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (vs[q] && b + q < nbins) {
-        if (kU64) atomicAdd(reinterpret_cast<unsigned long long*>(p.out) + orow + b + q, (unsigned long long)vs[q]);
-        else atomicAdd(reinterpret_cast<uint32_t*>(p.out) + orow + b + q, vs[q]);
-      }
-    }
-  }
-}
 
 // ------------------------------------------------------------------------------------------------
 // Split form of the same step-4 work (the default): the parity phase of every pair runs in its own

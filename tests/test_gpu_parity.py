@@ -397,3 +397,33 @@ def test_lonlat_vertices_exactly_on_centres(cuda_device):
     t = device_raster(spec, rows, cols)
     for tile in (16, 64, 100, 128, 704):
         assert (gpu_hist(t, gt, P, 256, tile, cols, nodata=-32768) == H).all(), tile
+
+
+@pytest.mark.parametrize("teeth", [700, 1600, 3500])
+@pytest.mark.parametrize("flip_x", [False, True])
+def test_comb_polygon_many_crossings(cuda_device, teeth, flip_x):
+    """A comb whose every tooth row is crossed by 2 x teeth edges: 1,400 crossings per row fit the
+    band kernel's shared flip list several rows at a time, 3,200 one row at a time, and 7,000
+    overflow it (the exact per-(pair, row) slow path of k_parity.cu).  Mirrored x (gt1 < 0) takes
+    the suffix form of the crossings.  GPU == literal O0."""
+    rows, cols = 48, 1024
+    gt = [0.0, 1.0, 0.0, float(rows), 0.0, -1.0]
+    if flip_x:
+        gt[0], gt[1] = float(cols), -1.0
+    xs, ys = [3.25], [4.5]
+    step = (cols - 8.0) / teeth
+    for i in range(teeth):
+        x0 = 4.0 + i * step
+        xs += [x0 + 0.1 * step, x0 + 0.3 * step, x0 + 0.6 * step, x0 + 0.9 * step]
+        ys += [4.5, 40.25, 40.25, 4.5]
+    xs += [cols - 3.5, cols - 3.5, 3.25]
+    ys += [4.5, 1.75, 1.75]
+    P = from_rings([[(np.array(xs), np.array(ys))], [(np.array([1.0, 900.0, 900.0, 1.0]),
+                                                       np.array([20.0, 20.0, 30.0, 30.0]))]])
+    spec = TINY.dem
+    R = fill_host(spec, cols, 0, 0, rows, cols)
+    H = oracle.o0(R, gt, P, oracle.make_bins(256, nodata=-32768), prefilter=True)
+    assert H[0].sum() > 0
+    t = device_raster(spec, rows, cols)
+    for tile in (16, 48, 256):
+        assert (gpu_hist(t, gt, P, 256, tile, cols, nodata=-32768) == H).all(), tile
