@@ -90,6 +90,12 @@ class ClockSampler:
         return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
 
 
+# BASELINE.json's metric (raster cells/s), measured over one device step; the end-to-end seconds
+# are the e2e / e2e_resident objects of the same line
+METRIC = ("raster cells/s (zonal histogram of the whole raster; device step = pairing + fused steps 1/3/4 "
+          "with raster and polygons resident in HBM; e2e objects: host-side end to end)")
+
+
 def measured_peaks() -> dict:
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -98,15 +104,17 @@ def measured_peaks() -> dict:
     return {"hbm_gbs": 6650.0, "source": "fallback (B200_PROFILING.md)"}
 
 
-def traffic_from_profile(kernel_key: str):
+def traffic_from_profile(kernel_key: str, config: str, tile: int, path: str):
     """dram read+write bytes per launch of the dominant kernel from the committed ncu --set full
-    summary (profiles/ncu_traffic.json), or None."""
+    capture of THIS configuration (profiles/ncu_traffic.json: {"<config>/T<tile>/<path>": {kernel:
+    bytes}}), or None when no capture of this configuration exists (another config's bytes would
+    say nothing about this launch)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
         return None
     try:
         d = json.load(open(p))
-        return d.get(kernel_key)
+        return d.get(f"{config}/T{tile}/{path}", {}).get(kernel_key)
     except Exception:
         return None
 
@@ -176,7 +184,7 @@ def run_reference(args, cfg):
     value = cells / (ms / 1000.0)
     sample = (f"rows [{start},{start + n}) x all {cfg.cols} cols of {cfg.name} ({cells} cells, "
               f"{P.n_poly} polygons), oracle O1 (row-hoisted Franklin test), {threads} threads")
-    line = {"impl": "reference", "metric": "raster cells/s (zonal histogram, end-to-end)", "value": value,
+    line = {"impl": "reference", "metric": METRIC, "value": value,
             "unit": "cells/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
             "data": "synthetic", "config": cfg.describe(),
@@ -227,7 +235,8 @@ def main():
     import torch.distributed as dist
 
     from paper_conf_ipps_zhangw14_b200 import zh
-    from paper_conf_ipps_zhangw14_b200.dist import SparseReducer, plan_shards, reduce_histograms, touched_polygons
+    from paper_conf_ipps_zhangw14_b200.dist import (SparseReducer, plan_shards, reduce_histograms, strip_polygons,
+                                                    touched_polygons)
     from synth.dem import fill_device
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -239,6 +248,10 @@ def main():
     if shared:
         local = 0
     torch.cuda.set_device(local)
+    if world > 1 and not shared:
+        # communicator set-up lines in the log (which NCCL transport / NVLS the ranks got)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     if world > 1:
         if shared:
             dist.init_process_group("gloo")
@@ -264,21 +277,37 @@ def main():
     log(f"raster shard rows [{r0},{r1}) generated ({time.perf_counter() - t_setup:.1f}s)")
     raster_v = raster[:nrows]
     out = torch.zeros((P.n_poly, cfg.nbins), dtype=torch.int64, device="cuda")
-    z = zh.ZonalHistogram(raster_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
+    # N > 1: each rank pairs only the polygons whose bounding box meets its strip (the others have
+    # no cell centre there); its rows land in the global [n_poly, nbins] buffer by one index copy
+    if world > 1:
+        ids = strip_polygons(P, cfg.gt, r0, r1)
+        Pr = P.subset(ids)
+        out_r = torch.zeros((max(len(ids), 1), cfg.nbins), dtype=torch.int64, device="cuda")[:len(ids)]
+        idx = torch.as_tensor(ids, device="cuda")
+        log(f"rank {rank}: rows [{r0},{r1}), {len(ids)} of {P.n_poly} polygons")
+    else:
+        ids, Pr, out_r, idx = None, P, out, None
+
+    def to_global():
+        if idx is not None and len(ids):
+            out.index_copy_(0, idx, out_r)
+
+    z = zh.ZonalHistogram(raster_v, cfg.gt, Pr, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
                           oor_drop=cfg.oor_drop, tile=T, rows=cfg.rows, cols=cfg.cols, row0=r0, stream=stream,
                           fused=(args.path == "fused"), cover=args.cover)
-    z.set_output(out)
+    z.set_output(out_r)
 
     # N > 1: sparse reduce (only polygons spanning strips are summed; the plan is geometry only),
     # unless --dense-reduce (the shared-GPU gloo mode stages its point-to-point rows through the host)
     reducer = None
     if world > 1 and not args.dense_reduce:
         z.zh_pair_tiles()
-        reducer = SparseReducer(touched_polygons(z), P.n_poly, device=out.device)
+        reducer = SparseReducer(ids[touched_polygons(z)], P.n_poly, device=out.device)
         log(f"sparse reduce: {len(reducer.shared)} shared polygons, {reducer.rows_moved()} rows moved "
             f"(dense: {world * P.n_poly})")
 
     def reduce_out():
+        to_global()
         if reducer is not None:
             reducer.reduce(out, to_rank0=True)
         else:
@@ -362,7 +391,8 @@ def main():
     else:
         kern["k_tile_hist"] = (avg(lib_ms, "step1_tile_hist"), 2.0 * cells_local + 4.0 * B_pad * st["n_tiles"])
         kern["k_aggregate"] = (avg(lib_ms, "step3_aggregate"), 4.0 * cfg.nbins * st["n_inside"])
-        kern["k_pip"] = (avg(lib_ms, "step4_pip_update"), 2.0 * st["n_isect"] * T * T)
+        kern["k_pip_cells+k_parity (pair-cell bytes, not HBM bytes)"] = (avg(lib_ms, "step4_pip_update"),
+                                                                         2.0 * st["n_isect"] * T * T)
         steps_detail = {"step2_pair_tiles": {"ms": avg(lib_ms, "step2_pair_tiles")}}
     for name, (t, b) in kern.items():
         steps_detail[name] = {"ms": t, "alg_bytes": b, "alg_GBps": b / (t / 1000.0) / 1e9 if t else None}
@@ -380,7 +410,7 @@ def main():
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / peaks["hbm_gbs"],
                 # the ncu capture is of the N = 1 launch; a shard's launch is a different one
-                "traffic": traffic_from_profile(dom) if world == 1 else None,
+                "traffic": traffic_from_profile(dom, cfg.name, T, path) if world == 1 else None,
                 "peak_source": peaks["source"], "alg_bytes_per_launch": dom_b,
                 "share_of_step": dom_ms / ms if ms > 0 else None}
     log(f"timed ({path}): {ms:.3f} ms/step, {steps_detail}")
@@ -409,18 +439,26 @@ def main():
                            ("step4_pip_update", 2.0 * st2["n_isect"] * T * T)):
                 t = avg(lib_ms, key)
                 other[key] = {"ms": t}
-                if b:
+                if b and key != "step4_pip_update":
                     other[key]["alg_GBps"] = b / (t / 1000.0) / 1e9 if t else None
                     other[key]["frac_of_hbm_peak"] = other[key]["alg_GBps"] / peaks["hbm_gbs"] if t else None
+                elif b:
+                    # 2 B x every cell of every intersecting pair: pairs sharing a tile re-read it
+                    # (from L2), and vectors with no inside cell are not read at all — a rate of
+                    # pair-cells, not of HBM bytes (ncu: profiles/ for the DRAM bytes)
+                    other[key]["pair_cell_GBps"] = b / (t / 1000.0) / 1e9 if t else None
         else:
             other["fused_update"] = {"ms": avg(lib_ms, "fused_update")}
         log(f"other path: {other}")
 
     # ---- end to end through the C ABI from host buffers
     e2e = None
+    e2e_res = None
     host = None
     if not args.no_e2e:
-        e2e, host = run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log, reduce_out)
+        e2e_res = run_e2e_resident(args, cfg, P, Pr, raster_v, out, out_r, r0, world, rank, stream, log, reduce_out)
+        e2e, host = run_e2e(args, cfg, P, Pr, z, raster_v, out, out_r, r0, nrows, pitch, world, rank, stream, log,
+                            reduce_out)
     z.close()
 
     cpu = None
@@ -437,7 +475,7 @@ def main():
 
     if rank == 0:
         clocks = clk.summary()
-        line = {"metric": "raster cells/s (zonal histogram, end-to-end)", "value": value, "unit": "cells/s",
+        line = {"metric": METRIC, "value": value, "unit": "cells/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
                 "data": "synthetic (fractal int16 DEM + jagged Voronoi counties, seeded)",
@@ -447,7 +485,7 @@ def main():
                                + ("" if world == 1 else (" sparse-reduce" if reducer is not None else " dense-reduce")),
                                l2="inputs larger than L2 (40 GB raster)", counts="uint64", pip="float64 no-FMA",
                                semantics="closed rectangle meets polygon (R15)" if args.cover else "centre inside"),
-                "e2e": e2e, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
+                "e2e": e2e, "e2e_resident": e2e_res, "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu,
                 "clocks": clocks, "path": path, "steps_detail": steps_detail, "other_path": other,
                 "pairs": {k: st[k] for k in ("n_tiles", "n_candidates", "n_inside", "n_isect", "n_band_entries",
                                              "n_edges", "n_pure_tiles", "n_pip_pairs", "n_pure_cells", "n_pip_cells")},
@@ -459,7 +497,79 @@ def main():
     return 0
 
 
-def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, stream, log, reduce_out):
+def _pin_polygons(P):
+    """Page-lock the polygon vertex arrays (zh_create's H2D then runs at PCIe speed)."""
+    import numpy as np
+    import torch
+    cudart = torch.cuda.cudart()
+    pinned = []
+    for a in (P.x, P.y):
+        if a.flags.c_contiguous and a.dtype == np.float64 and a.nbytes:
+            rv = cudart.cudaHostRegister(a.ctypes.data, a.nbytes, 0)
+            if (int(rv) if not isinstance(rv, tuple) else int(rv[0])) == 0:
+                pinned.append(a)
+    return pinned
+
+
+def _unpin(arrs):
+    import torch
+    for a in arrs:
+        torch.cuda.cudart().cudaHostUnregister(a.ctypes.data)
+
+
+def run_e2e_resident(args, cfg, P, Pr, raster_v, out, out_r, r0, world, rank, stream, log, reduce_out):
+    """SURVEY.md §8d's end-to-end time (the paper's, §IV.A: data resident in GPU memory,
+    disk I/O excluded): from "raster in HBM, polygons on the host" to "P x B matrix on the host" —
+    zh_create (polygon H2D), zh_run (step 2 + fused steps 1/3/4), the reduce (N > 1), the result
+    D2H and zh_destroy, every step."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangw14_b200 import zh
+    poly_pinned = _pin_polygons(Pr)
+    res_pin = torch.empty((P.n_poly, cfg.nbins), dtype=torch.int64, pin_memory=True)
+    res = res_pin.numpy().view(np.uint64)
+    times = []
+    for it in range(max(args.e2e_steps, 5) + 1):  # first iteration is a warm-up
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        z2 = zh.ZonalHistogram(raster_v, cfg.gt, Pr, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
+                               oor_drop=cfg.oor_drop, tile=cfg.tile, rows=cfg.rows, cols=cfg.cols, row0=r0,
+                               stream=stream, fused=(args.path == "fused"), cover=args.cover)
+        if world > 1:
+            z2.set_output(out_r)
+            z2.zh_run(None)
+            reduce_out()
+            if rank == 0:
+                res_pin.copy_(out, non_blocking=True)
+            torch.cuda.synchronize()
+        else:
+            z2.zh_run(res)
+        dt = time.perf_counter() - t0
+        z2.close()
+        t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        if it > 0:
+            times.append(float(t.item()))
+    _unpin(poly_pinned)
+    sec = sum(times) / len(times)
+    h2d = Pr.x.nbytes + Pr.y.nbytes + Pr.poly_ring_off.nbytes // 2 + Pr.ring_vert_off.nbytes // 2
+    if world > 1:
+        h2d_t = torch.tensor([h2d], dtype=torch.int64, device="cuda")
+        dist.all_reduce(h2d_t)
+        h2d = int(h2d_t.item())
+    log(f"e2e (resident raster) {sec:.4f} s/step")
+    return {"value": cfg.cells / sec, "unit": "cells/s", "seconds_per_step": sec, "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": P.n_poly * cfg.nbins * 8, "steps": len(times),
+            "includes": "raster resident in HBM (SURVEY.md 8d / PAPER.md:22): zh_create (polygon H2D from pinned "
+                        "host arrays) + zh_run (step 2 + fused update) + reduce (N > 1) + result D2H + zh_destroy"}
+
+
+def run_e2e(args, cfg, P, Pr, z, raster_v, out, out_r, r0, nrows, pitch, world, rank, stream, log, reduce_out):
     """E2E through the public API: host raster (pinned) + host polygons -> host histogram."""
     import numpy as np
     import torch
@@ -476,12 +586,7 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
     torch.from_numpy(host)[:nrows].copy_(raster_v)
     # the polygon vertex arrays are pinned too (zh_create's H2D of 154 MB then runs at PCIe speed
     # instead of through pageable staging)
-    poly_pinned = []
-    for a in (P.x, P.y):
-        if a.flags.c_contiguous and a.dtype == np.float64 and a.nbytes:
-            rv = cudart.cudaHostRegister(a.ctypes.data, a.nbytes, 0)
-            if (int(rv) if not isinstance(rv, tuple) else int(rv[0])) == 0:
-                poly_pinned.append(a)
+    poly_pinned = _pin_polygons(Pr)
     torch.cuda.synchronize()
     z.close()  # free the resident context's tile histograms before the e2e context allocates its own
     res_pin = torch.empty((P.n_poly, cfg.nbins), dtype=torch.int64, pin_memory=True)
@@ -493,11 +598,11 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
             dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        z2 = zh.ZonalHistogram(host_v, cfg.gt, P, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
+        z2 = zh.ZonalHistogram(host_v, cfg.gt, Pr, cfg.nbins, lo=cfg.lo, width=cfg.width, nodata=cfg.nodata,
                                oor_drop=cfg.oor_drop, tile=cfg.tile, rows=cfg.rows, cols=cfg.cols, row0=r0,
                                stream=stream, fused=(args.path == "fused"), cover=args.cover)
         if world > 1:
-            z2.set_output(out)
+            z2.set_output(out_r)
             z2.zh_run(None)
             reduce_out()
             if rank == 0:
@@ -515,11 +620,10 @@ def run_e2e(args, cfg, P, z, raster_v, out, r0, nrows, pitch, world, rank, strea
             times.append(float(t.item()))
     if pinned:
         cudart.cudaHostUnregister(host.ctypes.data)
-    for a in poly_pinned:
-        cudart.cudaHostUnregister(a.ctypes.data)
+    _unpin(poly_pinned)
     host = host[:nrows, :cfg.cols]
     sec = sum(times) / len(times)
-    poly_bytes = P.x.nbytes + P.y.nbytes + P.poly_ring_off.nbytes // 2 + P.ring_vert_off.nbytes // 2
+    poly_bytes = Pr.x.nbytes + Pr.y.nbytes + Pr.poly_ring_off.nbytes // 2 + Pr.ring_vert_off.nbytes // 2
     h2d = raster_h2d + poly_bytes  # the fused zh_run uploads only the tiles some pair needs
     if world > 1:
         h2d_total = torch.tensor([h2d], dtype=torch.int64, device="cuda")

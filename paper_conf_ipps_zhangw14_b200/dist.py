@@ -35,6 +35,30 @@ def plan_shards(rows: int, cols: int, gt, polygons, tile: int, world: int, balan
     return [int(b) for b in bounds]
 
 
+def strip_polygons(polygons, gt, r0: int, r1: int, margin: int = 2):
+    """Ids of the polygons whose vertex bounding box comes within `margin` rows of the strip's rows
+    [r0, r1): every other polygon has no cell centre in the strip (a centre inside a polygon lies
+    inside its bounding box), so its partial histogram on this strip is zero and the rank need not
+    pair it at all (step 2 over the strip's polygons only).  Host-side geometry,
+    computed once per decomposition."""
+    import numpy as np
+    P = polygons
+    if r1 <= r0 or P.n_poly == 0:
+        return np.zeros(0, dtype=np.int64)
+    first = P.ring_vert_off[P.poly_ring_off[:-1]]
+    last = P.ring_vert_off[P.poly_ring_off[1:]]
+    v = (np.asarray(P.y, dtype=np.float64) - gt[3]) / gt[5]  # fractional row coordinate
+    nonempty = np.nonzero(last > first)[0]
+    if nonempty.size == 0:
+        return np.zeros(0, dtype=np.int64)
+    lo = np.minimum.reduceat(v, first[nonempty])
+    hi = np.maximum.reduceat(v, first[nonempty])
+    # reduceat over the first vertex of each non-empty polygon: the segments run to the next
+    # non-empty polygon's first vertex, which is exactly this polygon's vertex range
+    keep = (hi >= r0 - margin) & (lo <= r1 + margin)
+    return nonempty[keep].astype(np.int64)
+
+
 def reduce_histograms(out, group=None, to_rank0: bool = False):
     """Sum the per-rank partial histograms in place.  `out` is the int64 (uint64 bits) or int32
     view of libzh's output; two's-complement sums are bit-identical to unsigned ones."""

@@ -155,3 +155,33 @@ def test_gloo_sparse_reduce_equals_single_process(world):
     n_shared = res[0][2]
     assert 0 < n_shared < P.n_poly  # some polygons span the strip borders, not all
     assert res[0][3] < world * P.n_poly  # fewer rows on the fabric than the dense reduce
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_strip_polygons_cover_every_nonzero_row(world):
+    """dist.strip_polygons: a rank that pairs only the polygons whose bounding box meets its strip
+    loses nothing — on every strip of the tiny and lon/lat configs the oracle's histograms of the
+    other polygons are all zero, and the strips' results summed equal the whole raster's."""
+    import oracle
+    from paper_conf_ipps_zhangw14_b200.dist import strip_polygons
+    from synth.configs import TINY, TINY_LONLAT
+    from synth.dem import fill_host
+    for cfg in (TINY, TINY_LONLAT):
+        P = cfg.polygons()
+        bins = oracle.make_bins(cfg.nbins, nodata=cfg.nodata)
+        R = fill_host(cfg.dem, cfg.cols, 0, 0, cfg.rows, cfg.cols)
+        whole = oracle.o1(R, cfg.gt, P, bins)
+        acc = np.zeros_like(whole)
+        for r in range(world):
+            r0, r1 = shard_rows(cfg.rows, 64, world, r)
+            ids = strip_polygons(P, cfg.gt, r0, r1)
+            H = oracle.o1(R[r0:r1], cfg.gt, P, bins, row0=r0)
+            others = np.setdiff1d(np.arange(P.n_poly), ids)
+            assert not H[others].any()
+            if r1 > r0:
+                Hs = oracle.o1(R[r0:r1], cfg.gt, P.subset(ids), bins, row0=r0)
+                assert (Hs == H[ids]).all()
+            acc += H
+        assert (acc == whole).all()
+        assert len(strip_polygons(P, cfg.gt, 0, cfg.rows)) == P.n_poly
+        assert len(strip_polygons(P, cfg.gt, 5, 5)) == 0
