@@ -213,6 +213,8 @@ def main():
     ap.add_argument("--path", default="fused", choices=["fused", "four_step"],
                     help="fused: step 2 + zh_fused_update (steps 1+3+4 fused, SURVEY §8f-1); four_step: 2,1,3,4")
     ap.add_argument("--no-other", action="store_true", help="skip timing the other path")
+    ap.add_argument("--no-graph", action="store_true",
+                    help="issue the step's calls one by one instead of replaying them from a CUDA graph (zh_step_graph)")
     ap.add_argument("--cover", action="store_true",
                     help="count cells whose closed rectangle meets the polygon (R15, PAPER.md:12) instead of "
                          "testing the cell centre (not the headline configuration)")
@@ -319,13 +321,16 @@ def main():
 
     def one_step(record=False, mode=None):
         mode = mode or path
-        z.zh_pair_tiles()
-        if mode == "fused":
-            z.zh_fused_update()
+        if mode == path and not args.no_graph:
+            z.zh_step_graph()  # the step replayed from a CUDA graph (captured during the warm-up)
         else:
-            z.zh_tile_hist()
-            z.zh_aggregate()
-            z.zh_pip_update()
+            z.zh_pair_tiles()
+            if mode == "fused":
+                z.zh_fused_update()
+            else:
+                z.zh_tile_hist()
+                z.zh_aggregate()
+                z.zh_pip_update()
         if record:
             lib_ms.append(z.step_ms())  # syncs after the step's last kernel
         if world > 1:

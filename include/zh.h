@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 6
+#define ZH_ABI_VERSION 7
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -186,6 +186,17 @@ zh_status zh_fused_update(zh_ctx ctx);
  * on_host with options.fused: the upload follows step 2 and covers only the needed tiles (see
  * zh_raster). */
 zh_status zh_run(zh_ctx ctx, void* host_out);
+
+/* One whole step — zh_pair_tiles + zh_fused_update (options.fused = 1), else zh_pair_tiles +
+ * zh_tile_hist + zh_aggregate + zh_pip_update — replayed from a CUDA graph.  The step's list sizes
+ * are a function of the context's fixed geometry: the first call runs the step directly and learns
+ * them (host syncs); the next call captures the step (on a context-owned stream) and every later
+ * call launches the captured graph: one launch, no host round trip.  A device check compares each
+ * replay's counts with the learnt sizes and any mismatch is reported (ZH_ERR_STATE) by the next
+ * syncing call.  Enqueued on options.stream, asynchronous; afterwards the histogram is complete
+ * as after the individual calls.  zh_set_output / zh_set_timing drop the captured graph.  Host
+ * rasters need zh_upload_raster (or a zh_run) first. */
+zh_status zh_step_graph(zh_ctx ctx);
 
 /* Device memory of destroyed contexts is kept in a process-wide cache and reused by later
  * contexts of the same device (no cudaMalloc / cudaFree of the raster copy per zh_create /

@@ -357,7 +357,7 @@ cudaError_t launch_fused(Ctx& c) {
   cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 6, c.stream);
   if (NT == 0 || NI + NX == 0) {
     if (c.timing)
-      for (int i = 10; i < 16; ++i) cudaEventRecord(c.ev[i], c.stream);
+      for (int i = 10; i < 16; ++i) rec_event(c, c.ev[i], c.stream);
     return cudaGetLastError();
   }
 
@@ -417,21 +417,27 @@ cudaError_t launch_fused(Ctx& c) {
   // exact grid for the cell kernel: the list sizes are copied to the host behind the list kernels
   // and read while the pure-tile kernel runs (no CTAs that only find they have no work)
   if ((e = pip_prepare(c, NI + NX)) != cudaSuccess) return e;
-  cudaMemcpyAsync(c.pinned_counts + 8, c.d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c.stream);
-  cudaEventRecord(c.ev_counts, c.stream);
+  if (!c.fused_known) {
+    cudaMemcpyAsync(c.pinned_counts + 8, c.d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c.stream);
+    cudaEventRecord(c.ev_counts, c.stream);
+  } else {  // known sizes (fixed geometry): the device checks the recomputed counts
+    const int64_t want[4] = {c.n_pip_known, 0, 0, c.n_grp_known};
+    if ((e = launch_check_counts(c, c.d_fcounts.as<int64_t>() + 1, want, 1)) != cudaSuccess) return e;
+    if ((e = launch_check_counts(c, c.d_fcounts.as<int64_t>() + 4, want + 3, 1)) != cudaSuccess) return e;
+  }
   auto parity = [&](int64_t grid) -> cudaError_t {
     cudaError_t pe;
-    if (c.timing) cudaEventRecord(c.ev[13], c.stream);
+    if (c.timing) rec_event(c, c.ev[13], c.stream);
     if ((pe = launch_parity(c, c.d_pip.as<int2>(), grid, c.d_fcounts.as<int64_t>() + 1, c.stream)) != cudaSuccess)
       return pe;
     if (c.cover) {  // R15: cells an edge reaches join the parity bits (k_touch.cu)
       if ((pe = launch_touch(c, c.d_remap.as<int32_t>(), c.stream)) != cudaSuccess) return pe;
     }
-    if (c.timing) cudaEventRecord(c.ev[14], c.stream);
+    if (c.timing) rec_event(c, c.ev[14], c.stream);
     return cudaSuccess;
   };
   // pure tiles: steps 1 + 3 fused (grid = upper bound, surplus CTAs exit at once)
-  if (c.timing) cudaEventRecord(c.ev[10], c.stream);
+  if (c.timing) rec_event(c, c.ev[10], c.stream);
   if (NI > 0) {
     const size_t smem = (size_t)hist_words(c.bp.nbins) * 4;
     const int run = pure_params(c).run;
@@ -456,24 +462,29 @@ cudaError_t launch_fused(Ctx& c) {
     c.launches += 1;
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
-  if (c.timing) cudaEventRecord(c.ev[11], c.stream);
-  if ((e = cudaEventSynchronize(c.ev_counts)) != cudaSuccess) return e;
-  const int64_t n_pip = c.pinned_counts[8 + 1];
-  const int64_t n_grp = c.pinned_counts[8 + 4];
+  if (c.timing) rec_event(c, c.ev[11], c.stream);
+  if (!c.fused_known) {
+    if ((e = cudaEventSynchronize(c.ev_counts)) != cudaSuccess) return e;
+    c.n_pip_known = c.pinned_counts[8 + 1];
+    c.n_grp_known = c.pinned_counts[8 + 4];
+    c.fused_known = true;
+  }
+  const int64_t n_pip = c.n_pip_known;
+  const int64_t n_grp = c.n_grp_known;
   if (n_pip > 0) {
     if ((e = parity(n_pip)) != cudaSuccess) return e;
   } else if (c.timing) {
-    cudaEventRecord(c.ev[13], c.stream);
-    cudaEventRecord(c.ev[14], c.stream);
+    rec_event(c, c.ev[13], c.stream);
+    rec_event(c, c.ev[14], c.stream);
   }
-  if (c.timing) cudaEventRecord(c.ev[15], c.stream);
+  if (c.timing) rec_event(c, c.ev[15], c.stream);
   if (grouped)
     e = n_grp > 0 ? launch_mixed_cells(c, c.d_pip.as<int2>(), c.d_pip_grp.as<int2>(), n_grp,
                                        c.d_fcounts.as<int64_t>() + 4)
                   : cudaSuccess;
   else
     e = n_pip > 0 ? launch_pip_cells(c, c.d_pip.as<int2>(), n_pip, c.d_fcounts.as<int64_t>() + 1) : cudaSuccess;
-  if (c.timing) cudaEventRecord(c.ev[12], c.stream);
+  if (c.timing) rec_event(c, c.ev[12], c.stream);
   return e;
 }
 

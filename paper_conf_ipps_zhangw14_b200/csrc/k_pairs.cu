@@ -329,6 +329,14 @@ __global__ void k_totals1(const int64_t* cand_off, const int64_t* band_base, int
   out[1] = band_base[P];
 }
 
+struct Want6 {
+  int64_t v[6];
+};
+__global__ void k_check_counts(const int64_t* __restrict__ counts, Want6 want, int n, uint32_t* __restrict__ flag) {
+  for (int i = 0; i < n; ++i)
+    if (counts[i] != want.v[i]) *flag = 1u;
+}
+
 static int grid_for(int64_t n, int threads) {
   int64_t b = (n + threads - 1) / threads;
   if (b > 148 * 32) b = 148 * 32;
@@ -351,6 +359,15 @@ static cudaError_t excl_scan(Ctx& c, const T* in, T* out, int64_t n) {
 
 
 namespace zh {
+
+cudaError_t launch_check_counts(Ctx& c, const int64_t* counts, const int64_t* want, int n) {
+  if (!c.d_flag.p) return cudaErrorInvalidValue;  // allocated and zeroed by zh_create
+  Want6 w = {};
+  for (int i = 0; i < n && i < 6; ++i) w.v[i] = want[i];
+  k_check_counts<<<1, 1, 0, c.stream>>>(counts, w, n < 6 ? n : 6, c.d_flag.as<uint32_t>());
+  c.launches += 1;
+  return cudaGetLastError();
+}
 
 cudaError_t launch_pairs_phase1(Ctx& c) {
   cudaError_t e;

@@ -342,6 +342,8 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   }
   if ((e = pinned_alloc((void**)&c->pinned_counts, &c->pinned_counts_bytes, 16 * sizeof(int64_t))) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create (pinned counters)"));
+  if ((e = c->d_flag.ensure(16)) != cudaSuccess || (e = cudaMemsetAsync(c->d_flag.p, 0, 16, c->stream)) != cudaSuccess)
+    return cleanup_fail(cuda_fail(e, "zh_create (check flag)"));
   for (int i = 0; i < 16; ++i)
     if ((e = cudaEventCreate(&c->ev[i])) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (events)"));
   if ((e = cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking)) != cudaSuccess ||
@@ -383,7 +385,7 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
                       &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats,
-                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_band_poly, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
+                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_band_poly, &c->d_flag, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
   for (auto* b : bufs) b->release();
   ZH_TR("release");
   for (int i = 0; i < 16; ++i)
@@ -393,6 +395,7 @@ extern "C" void zh_destroy(zh_ctx h) {
     cudaStreamSynchronize(c->side);
     cudaStreamDestroy(c->side);
   }
+  if (c->gexec) cudaGraphExecDestroy(c->gexec);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->ev_counts) cudaEventDestroy(c->ev_counts);
@@ -411,17 +414,28 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
                             &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats,
-                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_band_poly, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
+                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_band_poly, &c.d_flag, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;
 }
 
 static void tic(Ctx* c, int step) {
-  if (c->timing) cudaEventRecord(c->ev[2 * step], c->stream);
+  if (c->timing) zh::rec_event(*c, c->ev[2 * step], c->stream);
 }
 static void toc(Ctx* c, int step) {
-  if (c->timing) cudaEventRecord(c->ev[2 * step + 1], c->stream);
+  if (c->timing) zh::rec_event(*c, c->ev[2 * step + 1], c->stream);
+}
+
+// After a sync point: did a step's counts differ from the context's known sizes?  (Never, for a
+// fixed geometry; the check guards the host-sync-free steps.)
+static zh_status check_flag(Ctx* c, const char* who) {
+  if (!c->d_flag.p) return ZH_OK;
+  ZH_CU(cudaMemcpyAsync(c->pinned_counts + 15, c->d_flag.p, 4, cudaMemcpyDeviceToHost, c->stream), who);
+  ZH_CU(cudaStreamSynchronize(c->stream), who);
+  if (*reinterpret_cast<uint32_t*>(c->pinned_counts + 15) != 0u)
+    return fail(ZH_ERR_STATE, "%s: a step's list sizes differ from the context's known sizes", who);
+  return ZH_OK;
 }
 
 extern "C" zh_status zh_upload_raster(zh_ctx h) {
@@ -498,23 +512,34 @@ extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect
   const size_t out_bytes = (size_t)c->P * c->bp.nbins * (c->out_u64 ? 8 : 4);
   ZH_CU(cudaMemsetAsync(c->d_out, 0, out_bytes, c->stream), "zh_pair_tiles (zero output)");
   ZH_CU(zh::launch_pairs_phase1(*c), "zh_pair_tiles (phase 1)");
-  ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_counts.p, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
-        "zh_pair_tiles (counts)");
-  ZH_CU(cudaStreamSynchronize(c->stream), "zh_pair_tiles (sync 1)");
-  c->n_cand = c->pinned_counts[0];
-  c->n_bands = c->pinned_counts[1];
-  c->n_band_entries = c->pinned_counts[2];
-  if (c->n_cand >= (1ll << 31) || c->n_bands >= (1ll << 31) || c->n_band_entries >= (1ll << 31) ||
-      c->n_band_entries < 0)
-    return fail(ZH_ERR_UNSUPPORTED, "pair lists exceed 2^31 entries");
-  ZH_CU(zh::launch_pairs_phase2(*c), "zh_pair_tiles (phase 2)");
-  ZH_CU(cudaMemcpyAsync(c->pinned_counts + 4, c->d_counts.as<int64_t>() + 4, 2 * sizeof(int64_t),
-                        cudaMemcpyDeviceToHost, c->stream),
-        "zh_pair_tiles (counts)");
-  toc(c, 1);
-  ZH_CU(cudaStreamSynchronize(c->stream), "zh_pair_tiles (sync 2)");
-  c->n_inside = c->pinned_counts[4];
-  c->n_isect = c->pinned_counts[5];
+  if (c->sizes_known) {
+    // the sizes are those of the first call (fixed geometry): no host round trip; the device
+    // checks the recomputed counts against them
+    ZH_CU(zh::launch_pairs_phase2(*c), "zh_pair_tiles (phase 2)");
+    const int64_t want[6] = {c->n_cand, c->n_bands, c->n_band_entries, 0, c->n_inside, c->n_isect};
+    ZH_CU(zh::launch_check_counts(*c, c->d_counts.as<int64_t>(), want, 3), "zh_pair_tiles (check)");
+    ZH_CU(zh::launch_check_counts(*c, c->d_counts.as<int64_t>() + 4, want + 4, 2), "zh_pair_tiles (check)");
+    toc(c, 1);
+  } else {
+    ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_counts.p, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
+          "zh_pair_tiles (counts)");
+    ZH_CU(cudaStreamSynchronize(c->stream), "zh_pair_tiles (sync 1)");
+    c->n_cand = c->pinned_counts[0];
+    c->n_bands = c->pinned_counts[1];
+    c->n_band_entries = c->pinned_counts[2];
+    if (c->n_cand >= (1ll << 31) || c->n_bands >= (1ll << 31) || c->n_band_entries >= (1ll << 31) ||
+        c->n_band_entries < 0)
+      return fail(ZH_ERR_UNSUPPORTED, "pair lists exceed 2^31 entries");
+    ZH_CU(zh::launch_pairs_phase2(*c), "zh_pair_tiles (phase 2)");
+    ZH_CU(cudaMemcpyAsync(c->pinned_counts + 4, c->d_counts.as<int64_t>() + 4, 2 * sizeof(int64_t),
+                          cudaMemcpyDeviceToHost, c->stream),
+          "zh_pair_tiles (counts)");
+    toc(c, 1);
+    ZH_CU(cudaStreamSynchronize(c->stream), "zh_pair_tiles (sync 2)");
+    c->n_inside = c->pinned_counts[4];
+    c->n_isect = c->pinned_counts[5];
+    c->sizes_known = true;
+  }
   c->have_pairs = true;
   if (n_inside) *n_inside = c->n_inside;
   if (n_isect) *n_isect = c->n_isect;
@@ -583,6 +608,72 @@ extern "C" zh_status zh_run(zh_ctx h, void* host_out) {
     ZH_CU(cudaMemcpyAsync(host_out, c->d_out, out_bytes, cudaMemcpyDeviceToHost, c->stream), "zh_run (D2H)");
   }
   ZH_CU(cudaStreamSynchronize(c->stream), "zh_run (sync)");
+  return check_flag(c, "zh_run");
+}
+
+// The step's calls (no upload, no D2H) on c->stream.
+static zh_status run_step_calls(zh_ctx h) {
+  Ctx* c = C(h);
+  zh_status s;
+  if ((s = zh_pair_tiles(h, nullptr, nullptr)) != ZH_OK) return s;
+  if (c->fused) return zh_fused_update(h);
+  if ((s = zh_tile_hist(h)) != ZH_OK) return s;
+  if ((s = zh_aggregate(h)) != ZH_OK) return s;
+  return zh_pip_update(h);
+}
+
+extern "C" zh_status zh_step_graph(zh_ctx h) {
+  if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
+  Ctx* c = C(h);
+  if (c->on_host && c->rp.nrows > 0 && c->h2d_bytes == 0)
+    return fail(ZH_ERR_STATE, "zh_step_graph on a host raster needs zh_upload_raster (or a zh_run) first");
+  // the first call runs the step directly: it learns the list sizes (host syncs)
+  if (!c->sizes_known || (c->fused && !c->fused_known)) return run_step_calls(h);
+  if (c->gexec && c->graph_fused != c->fused) {
+    cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+  }
+  if (!c->gexec) {
+    // capture on the context's own non-blocking stream (the caller's stream may be the legacy
+    // default stream, which cannot be captured); the launches below fork/join it to c->stream
+    cudaStream_t user = c->stream;
+    ZH_CU(cudaStreamBeginCapture(c->side, cudaStreamCaptureModeThreadLocal), "zh_step_graph (capture)");
+    c->stream = c->side;
+    c->capturing = true;
+    const int64_t before = c->launches;
+    const zh_status st = run_step_calls(h);
+    c->graph_kernels = c->launches - before;  // kernel nodes of the graph (recorded, not launched)
+    c->launches = before;
+    c->stream = user;
+    c->capturing = false;
+    cudaGraph_t g = nullptr;
+    const cudaError_t e = cudaStreamEndCapture(c->side, &g);
+    if (st != ZH_OK) {
+      if (g) cudaGraphDestroy(g);
+      return st;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "zh_step_graph (end capture)");
+    const cudaError_t ei = cudaGraphInstantiate(&c->gexec, g, 0);
+    cudaGraphDestroy(g);
+    if (ei != cudaSuccess) {
+      c->gexec = nullptr;
+      return cuda_fail(ei, "zh_step_graph (instantiate)");
+    }
+    c->graph_fused = c->fused;
+  }
+  ZH_CU(cudaEventRecord(c->ev_fork, c->stream), "zh_step_graph");
+  ZH_CU(cudaStreamWaitEvent(c->side, c->ev_fork, 0), "zh_step_graph");
+  ZH_CU(cudaGraphLaunch(c->gexec, c->side), "zh_step_graph (launch)");
+  ZH_CU(cudaEventRecord(c->ev_join, c->side), "zh_step_graph");
+  ZH_CU(cudaStreamWaitEvent(c->stream, c->ev_join, 0), "zh_step_graph");
+  c->launches += c->graph_kernels;
+  c->have_pairs = true;
+  if (c->fused) {
+    c->fused_done = true;
+  } else {
+    c->have_hist = true;
+    c->step3_done = c->step4_done = true;
+  }
   return ZH_OK;
 }
 
@@ -758,6 +849,10 @@ extern "C" zh_status zh_set_output(zh_ctx h, void* dptr) {
   Ctx* c = C(h);
   if (dptr && ((uintptr_t)dptr & 7u)) return fail(ZH_ERR_INVALID_ARG, "output buffer must be 8-byte aligned");
   c->d_out = dptr ? dptr : c->d_out_own.p;
+  if (c->gexec) {  // the captured step writes the old buffer
+    cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+  }
   c->have_pairs = false;  // the new buffer must be zeroed by zh_pair_tiles before accumulation
   c->have_hist = c->have_hist;
   return ZH_OK;
@@ -802,6 +897,8 @@ extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
   s->device_bytes = (int64_t)zh::device_bytes(*c);
   s->h2d_bytes = c->h2d_bytes;
   s->n_pure_tiles = s->n_pip_pairs = s->n_pure_cells = s->n_pip_cells = s->n_mixed_groups = s->n_group_cells = 0;
+  zh_status fs = check_flag(c, "zh_get_stats");
+  if (fs != ZH_OK) return fs;
   if (c->fused_done) {
     ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
           "zh_get_stats");
@@ -818,7 +915,12 @@ extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
 
 extern "C" zh_status zh_set_timing(zh_ctx h, int32_t enable) {
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
-  C(h)->timing = enable != 0;
+  Ctx* c = C(h);
+  if (c->gexec && c->timing != (enable != 0)) {  // the captured step records (or not) the events
+    cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+  }
+  c->timing = enable != 0;
   return ZH_OK;
 }
 
@@ -826,7 +928,10 @@ extern "C" zh_status zh_get_step_ms(zh_ctx h, float* ms, int32_t n) {
   if (!h || !ms) return fail(ZH_ERR_INVALID_ARG, "null argument");
   Ctx* c = C(h);
   if (!c->timing) return fail(ZH_ERR_STATE, "timing is disabled");
-  ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_step_ms");
+  {
+    zh_status fs = check_flag(c, "zh_get_step_ms");
+    if (fs != ZH_OK) return fs;
+  }
   // (start, stop) event pairs: steps 1..4, fused, fused pure-tile kernel, fused cell-in-polygon
   // (cell) kernel, fused parity kernel (second stream, overlapping the pure-tile kernel)
   const int pairs[8][2] = {{0, 1}, {2, 3}, {4, 5}, {6, 7}, {8, 9}, {10, 11}, {15, 12}, {13, 14}};

@@ -93,7 +93,25 @@ struct Ctx {
   uint8_t* pinned_need = nullptr;       // on_host + fused zh_run: per-tile 'needed' flags (host copy)
   size_t pinned_counts_bytes = 0, pinned_need_bytes = 0;  // sizes of the cached pinned blocks
   DBuf d_need;
+  // Sizes of the step's lists are a function of the context's fixed geometry (polygons, raster
+  // extent, tile): the first zh_pair_tiles / zh_fused_update learn them with host syncs, later calls
+  // reuse them and run with no host round trip (capturable in a CUDA graph, zh_step_graph); a
+  // device check (k_check_counts) flags any step whose counts differ, reported at the next sync.
+  bool sizes_known = false, fused_known = false;
+  int64_t n_pip_known = 0, n_grp_known = 0;
+  DBuf d_flag;
+  bool capturing = false;                 // recording a CUDA graph: events become external records
+  cudaGraphExec_t gexec = nullptr;
+  int32_t graph_fused = -1;               // the path the graph was captured for
+  int64_t graph_kernels = 0;              // kernel launches one replay performs
 };
+
+// Timing event on stream s (an external record node while a graph is being captured).
+inline void rec_event(const Ctx& c, cudaEvent_t e, cudaStream_t s) {
+  cudaEventRecordWithFlags(e, s, c.capturing ? cudaEventRecordExternal : cudaEventRecordDefault);
+}
+// Device check of counts[i] == want[i] (i < n <= 6); sets *flag (k_pairs.cu).
+cudaError_t launch_check_counts(Ctx& c, const int64_t* counts, const int64_t* want, int n);
 
 // kernels / launchers (k_*.cu)
 cudaError_t launch_tile_hist(Ctx& c);

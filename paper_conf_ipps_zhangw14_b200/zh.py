@@ -67,7 +67,7 @@ class zh_stats(ctypes.Structure):
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",
            "zh_fused_update", "zh_zonal_stats", "zh_zonal_summary", "zh_hist_distance", "zh_plan_rows",
-           "zh_run", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
+           "zh_run", "zh_step_graph", "zh_output_device", "zh_set_output", "zh_copy_tile_hist", "zh_copy_pairs", "zh_get_stats",
            "zh_set_timing", "zh_get_step_ms", "zh_launch_count", "zh_last_error", "zh_abi_version", "zh_destroy",
            "zh_trim_cache", "zh_cache_bytes"]
 
@@ -94,6 +94,7 @@ def _load():
         "zh_plan_rows": (st, [ctypes.POINTER(zh_raster), ctypes.POINTER(zh_polygons), ctypes.POINTER(zh_options), i32,
                               vp, vp]),
         "zh_run": (st, [vp, vp]),
+        "zh_step_graph": (st, [vp]),
         "zh_output_device": (st, [vp, ctypes.POINTER(vp), ctypes.POINTER(i64)]),
         "zh_set_output": (st, [vp, vp]),
         "zh_copy_tile_hist": (st, [vp, vp, i64]),
@@ -261,6 +262,9 @@ class ZonalHistogram:
             return host_out
         _check(LIB.zh_run(self.h, None))
         return None
+
+    def zh_step_graph(self):
+        _check(LIB.zh_step_graph(self.h))
 
     def run(self) -> np.ndarray:
         out = np.empty((self.n_poly, self.nbins), dtype=np.uint64 if self.out_u64 else np.uint32)

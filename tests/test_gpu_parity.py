@@ -427,3 +427,30 @@ def test_comb_polygon_many_crossings(cuda_device, teeth, flip_x):
     t = device_raster(spec, rows, cols)
     for tile in (16, 48, 256):
         assert (gpu_hist(t, gt, P, 256, tile, cols, nodata=-32768) == H).all(), tile
+
+
+@pytest.mark.parametrize("fused", [True, False])
+def test_step_graph_replays(tiny, cuda_device, fused):
+    """zh_step_graph: first call direct (learns the sizes), second captures, later calls replay the
+    CUDA graph — every result equals the oracle; timing events work inside the graph; a new output
+    buffer drops the graph and the next replay writes the new buffer."""
+    import torch
+    zh = _zh()
+    cfg, P, R, H = tiny
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=cfg.tile, cols=cfg.cols, nodata=cfg.nodata,
+                           fused=fused) as z:
+        z.set_timing(True)
+        for i in range(4):
+            z.zh_step_graph()
+            got = z.output_device().cpu().numpy().view(np.uint64)
+            assert (got == H).all(), i
+            ms = z.step_ms()
+            assert ms["step2_pair_tiles"] > 0
+        out2 = torch.zeros((P.n_poly, cfg.nbins), dtype=torch.int64, device="cuda")
+        z.set_output(out2)
+        for i in range(3):
+            z.zh_step_graph()
+            assert (out2.cpu().numpy().view(np.uint64) == H).all(), i
+        st = z.stats()  # a syncing call: also checks the device count guard
+        assert st["n_isect"] > 0
