@@ -5,10 +5,10 @@
 // test on the CPU "using well-established computational geometry libraries", then Thrust
 // stable_sort_by_key / stable_partition / reduce_by_key / scan to build per-polygon segments.
 // B200 design, all on the GPU:
-//   1. k_edges   — one CTA per polygon, one thread per vertex: the ring edge it starts, in canonical orientation, and
-//                  the exact half-open interval of centre rows it straddles (ya <= yc(r) < yb),
+//   1. k_mbb_edges — one CTA per polygon: vertex MBB -> covered tile rectangle (1-cell margin);
+//                  then one thread per vertex: the ring edge it starts, in canonical orientation,
+//                  and the exact half-open interval of centre rows it straddles (ya <= yc(r) < yb),
 //                  found with the same yc(r) expression the PIP test uses;
-//   2. k_mbb     — one CTA per polygon: vertex MBB -> covered tile rectangle (1-cell margin);
 //   3. scans     — candidate offsets and band (polygon, tile-row) bases (CUB);
 //   4. k_poly_bands — per (polygon, tile row) lists of the edges whose row interval meets it (the
 //                  step-4 edge lists and the classifier's input), counted in shared memory;
@@ -67,14 +67,10 @@ __device__ __forceinline__ int2 straddle_rows(const Geo& g, double ya, double yb
 // (edge, tile row) band entries is added to *n_entries.  Polygons whose tile rectangle misses the
 // shard (empty MBB) are skipped: nothing downstream reads their edges.  (Rings are contiguous, so
 // no search is needed.)
-__global__ void __launch_bounds__(256) k_edges(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
-                                               const double* __restrict__ x, const double* __restrict__ y, Geo g,
-                                               int64_t rA, int64_t rB, int T, const int4* __restrict__ mbb,
-                                               Edge* __restrict__ edges, int2* __restrict__ erows,
-                                               int64_t* __restrict__ n_entries) {
-  const int k = blockIdx.x;
-  const int4 m = mbb[k];
-  if (m.x > m.y) return;
+__device__ __forceinline__ void edges_body(int k, const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                           const double* __restrict__ x, const double* __restrict__ y, const Geo& g,
+                                           int64_t rA, int64_t rB, int T, Edge* __restrict__ edges,
+                                           int2* __restrict__ erows, int64_t* __restrict__ n_entries) {
   int span = 0;
   for (int ring = pro[k]; ring < pro[k + 1]; ++ring) {
     const int a = rvo[ring], b = rvo[ring + 1];
@@ -95,13 +91,13 @@ __global__ void __launch_bounds__(256) k_edges(const int32_t* __restrict__ pro, 
                                                  (unsigned long long)span);
 }
 
-// One CTA per polygon: MBB of its vertices -> covered tile rectangle (global tile indices),
-// clipped to the raster columns and the shard rows.  Empty -> (1, 0, 1, 0).
-__global__ void __launch_bounds__(256) k_mbb(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
-                                              const double* __restrict__ x, const double* __restrict__ y, Geo g,
-                                              RasterP rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
-                                              int64_t* __restrict__ nband) {
-  const int k = blockIdx.x;
+// MBB of polygon k's vertices -> covered tile rectangle (global tile indices), clipped to the raster
+// columns and the shard rows.  Empty -> (1, 0, 1, 0).  Returned to every thread of the CTA.
+__device__ __forceinline__ int4 mbb_body(int k, const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                         const double* __restrict__ x, const double* __restrict__ y, const Geo& g,
+                                         const RasterP& rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
+                                         int64_t* __restrict__ nband) {
+  __shared__ int4 s_m;
   const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
   double xmn = INFINITY, xmx = -INFINITY, ymn = INFINITY, ymx = -INFINITY;
   for (int i = vb + threadIdx.x; i < ve; i += blockDim.x) {
@@ -146,7 +142,25 @@ __global__ void __launch_bounds__(256) k_mbb(const int32_t* __restrict__ pro, co
     mbb[k] = m;
     ncand[k] = nc;
     nband[k] = nb;
+    s_m = m;
   }
+  __syncthreads();
+  return s_m;
+}
+
+// One CTA per polygon (step 2, first pass): the MBB's tile rectangle, then — when it meets the
+// shard — the canonical edges and their exact straddled rows (the vertices are read twice, the
+// second time from L1/L2).
+__global__ void __launch_bounds__(256) k_mbb_edges(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
+                                                   const double* __restrict__ x, const double* __restrict__ y, Geo g,
+                                                   RasterP rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
+                                                   int64_t* __restrict__ nband, int64_t rA, int64_t rB,
+                                                   Edge* __restrict__ edges, int2* __restrict__ erows,
+                                                   int64_t* __restrict__ n_entries) {
+  const int k = blockIdx.x;
+  const int4 m = mbb_body(k, pro, rvo, x, y, g, rp, mbb, ncand, nband);
+  if (m.x > m.y) return;
+  edges_body(k, pro, rvo, x, y, g, rA, rB, rp.T, edges, erows, n_entries);
 }
 
 // Band lists, one CTA per polygon: its vertices (= edges) are contiguous, and the counters of its
@@ -386,15 +400,10 @@ cudaError_t launch_pairs_phase1(Ctx& c) {
   cudaMemsetAsync(c.d_nband.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
   cudaMemsetAsync(c.d_counts.p, 0, sizeof(int64_t) * 8, c.stream);
   if (P > 0) {
-    k_mbb<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
-                                   c.d_y.as<double>(), c.geo, c.rp, c.d_mbb.as<int4>(), c.d_ncand.as<int64_t>(),
-                                   c.d_nband.as<int64_t>());
-    c.launches += 1;
-  }
-  if (V > 0) {
-    k_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
-                                     c.d_y.as<double>(), c.geo, rA, rB, c.rp.T, c.d_mbb.as<int4>(),
-                                     c.d_edges.as<Edge>(), c.d_erows.as<int2>(), c.d_counts.as<int64_t>() + 2);
+    k_mbb_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
+                                         c.d_y.as<double>(), c.geo, c.rp, c.d_mbb.as<int4>(), c.d_ncand.as<int64_t>(),
+                                         c.d_nband.as<int64_t>(), rA, rB, c.d_edges.as<Edge>(), c.d_erows.as<int2>(),
+                                         c.d_counts.as<int64_t>() + 2);
     c.launches += 1;
   }
   if ((e = excl_scan<int64_t>(c, c.d_ncand.as<int64_t>(), c.d_cand_off.as<int64_t>(), P + 1)) != cudaSuccess) return e;

@@ -7,6 +7,9 @@
 #ifndef ZH_MIX_ROWS4
 #define ZH_MIX_ROWS4 1
 #endif
+#ifndef ZH_MIX_NR
+#define ZH_MIX_NR 4  // rows (16-byte loads) in flight per thread in k_mixed_cells' main loop
+#endif
 // k_mixed_cells: the two staged parity bitmaps interleaved word by word ({A word, B word} pairs), so
 // that one 8-byte shared load gives a vector's bits of both pairs.
 #ifndef ZH_MIX_IL
@@ -336,12 +339,13 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
         int lr = rs;
         if (!kO) {
 #if ZH_MIX_ROWS4
-          // four rows per iteration: four 16-byte loads in flight per thread
-          for (; lr + 3 * rpi < ch; lr += 4 * rpi, ptr += 4 * step) {
-            uint32_t e[4], s[4];
-            uint4 q[4];
+          // ZH_MIX_NR rows per iteration: that many 16-byte loads in flight per thread
+          constexpr int NR = ZH_MIX_NR;
+          for (; lr + (NR - 1) * rpi < ch; lr += NR * rpi, ptr += NR * step) {
+            uint32_t e[NR], s[NR];
+            uint4 q[NR];
 #pragma unroll
-            for (int u = 0; u < 4; ++u) {
+            for (int u = 0; u < NR; ++u) {
               const uint2 b2 = pb2(lr + u * rpi);
               e[u] = b2.y;
               s[u] = cskip | (~(b2.x | b2.y) & 0xFFu);
@@ -349,7 +353,7 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
               if (s[u] != 0xFFu) q[u] = ld_stream16(ptr + u * step);
             }
 #pragma unroll
-            for (int u = 0; u < 4; ++u)
+            for (int u = 0; u < NR; ++u)
               if (s[u] != 0xFFu) count_sel(q[u], s[u], e[u]);
           }
 #endif

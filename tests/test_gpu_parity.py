@@ -361,7 +361,7 @@ def test_lonlat_vertices_exactly_on_centres(cuda_device):
     """Non-dyadic equality cases: a 1-arc-second lon/lat geotransform with polygon
     vertices placed EXACTLY on computed cell centres — x = gt0 + (c + 0.5) gt1, y = gt3 + (r + 0.5) gt5,
     the same binary64 expressions both sides evaluate — so centre rows meet vertices (ya == yc: the
-    half-open straddle rule at its boundary, k_edges' exact row intervals), vertical edges sit on
+    half-open straddle rule at its boundary, k_mbb_edges' exact row intervals), vertical edges sit on
     centre columns (xi == xc: not a crossing) and shared borders pass through centres.  GPU ==
     literal O0 (no prefilter) at several tile sizes, both paths."""
     ARC = 1.0 / 3600.0

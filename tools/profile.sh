@@ -9,7 +9,7 @@ TAG=${1:-r02}
 mkdir -p gpurun_out
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_${TAG}.csv \
     python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu > gpurun_out/launches_${TAG}.log 2>&1
-K='k_tile_hist|k_aggregate|k_parity|k_pip_cells|k_fused_pure|k_mixed_cells|k_edges|k_classify|k_mark|k_poly_bands|k_mbb'
+K='k_tile_hist|k_aggregate|k_parity|k_pip_cells|k_fused_pure|k_mixed_cells|k_mbb_edges|k_classify|k_mark|k_poly_bands'
 for spec in "conus 256 fused" "conus 256 four_step" "state 256 fused" "pip-stress 256 fused"; do
   set -- $spec
   timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"$K" -c 12 \
@@ -21,7 +21,7 @@ for spec in "conus 256 fused" "conus 256 four_step" "state 256 fused" "pip-stres
   set -- $spec
   R=gpurun_out/full_${TAG}_$1_$3.ncu-rep
   { python tools/ncu_summary.py $R
-    for k in k_fused_pure k_mixed_cells k_parity k_tile_hist k_aggregate k_pip_cells k_edges k_classify; do
+    for k in k_fused_pure k_mixed_cells k_parity k_tile_hist k_aggregate k_pip_cells k_mbb_edges k_classify; do
       echo "### $k"; python tools/src_hotspots.py $R $k 12 2>/dev/null; done; } > gpurun_out/ncu_full_${TAG}_$1_$3.txt
   ZH_TRAFFIC_JSON=gpurun_out/ncu_traffic_${TAG}.json python tools/ncu_traffic.py $R $1 $2 $3
 done
