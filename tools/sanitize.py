@@ -1,5 +1,6 @@
 """Small end-to-end runs for compute-sanitizer (memcheck / racecheck / synccheck): tiny config,
-both paths, a ragged tile size, and the zonal statistics.  python tools/sanitize.py"""
+both paths, a ragged tile size, the CUDA-graph step, the zonal statistics / summary and the
+histogram distances (pair lists and all pairs, both product widths).  python tools/sanitize.py"""
 import os
 import sys
 
@@ -19,6 +20,19 @@ for tile, fused in ((128, False), (128, True), (100, True), (100, False)):
     with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=tile, nodata=cfg.nodata, fused=fused) as z:
         res.append(z.run())
         z.zh_zonal_stats()
+        z.zh_zonal_summary()
+        for kind in ("l1", "emd", "chi2"):
+            z.zh_hist_distance(kind)
+            z.zh_hist_distance(kind, [0, 3, 15], [1, 3, 2])
+        for _ in range(3):  # direct, captured, replayed
+            z.zh_step_graph()
+        res.append(z.output_device().cpu().numpy().view(np.uint64).copy())
+os.environ["ZH_DIST_WIDE"] = "1"
+with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=128, nodata=cfg.nodata) as z:
+    z.run()
+    for kind in ("l1", "emd", "chi2"):
+        z.zh_hist_distance(kind)
+del os.environ["ZH_DIST_WIDE"]
 assert all((r == res[0]).all() for r in res)
 cov = []
 for tile, fused in ((128, True), (100, False)):  # cover mode (R15): k_touch on top of the split step 4
