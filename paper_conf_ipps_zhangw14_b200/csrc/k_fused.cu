@@ -207,13 +207,24 @@ __device__ __forceinline__ void pure_flush(const PureP& f, int tile, const uint3
 #endif
 constexpr int kPureRun = ZH_PURE_RUN;
 
+constexpr int kPureRunMax = 256;  // pure_params caps the run at this many tiles
+
 template <int kMode, bool kU64>
 __global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
   const int64_t n = f.counts[0];
   const int64_t i0 = (int64_t)blockIdx.x * f.run;
   if (i0 >= n) return;
-  const int64_t i1 = min(n, i0 + (int64_t)f.run);
+  const int nrun = (int)(min(n, i0 + (int64_t)f.run) - i0);
   extern __shared__ __align__(16) uint32_t sh[];
+  // the run's tiles and where its inside-polygon set changes (a flush), decided by all threads at
+  // once: the per-tile list reads are one round of latency per CTA instead of one per tile
+  __shared__ int s_tile[kPureRunMax];
+  __shared__ uint8_t s_flush[kPureRunMax];
+  for (int j = threadIdx.x; j < nrun; j += blockDim.x) {
+    const int t = f.pure_tiles[i0 + j];
+    s_tile[j] = t;
+    s_flush[j] = (j == nrun - 1 || !same_polys(f, t, f.pure_tiles[i0 + j + 1])) ? 1 : 0;
+  }
   const int HW = hist_words(f.bp.nbins);
   auto zero = [&]() {
     for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
@@ -221,21 +232,19 @@ __global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
   };
   zero();
   __syncthreads();
-  int tile = f.pure_tiles[i0];
-  for (int64_t idx = i0; idx < i1; ++idx) {
+  for (int j = 0; j < nrun; ++j) {
+    const int tile = s_tile[j];
     const int trl = tile / f.rp.TC, tc = tile - trl * f.rp.TC;
     tile_histogram<kMode>(sh, f.rp, f.bp, f.fb, trl, tc);
-    const int next = idx + 1 < i1 ? f.pure_tiles[idx + 1] : -1;
-    if (next < 0 || !same_polys(f, tile, next)) {  // uniform over the CTA
+    if (s_flush[j]) {  // uniform over the CTA
       __syncthreads();
       pure_flush<kU64>(f, tile, sh);
-      if (next >= 0) {
+      if (j + 1 < nrun) {
         __syncthreads();
         zero();
         __syncthreads();
       }
     }
-    tile = next;
   }
 }
 
@@ -309,7 +318,7 @@ static PureP pure_params(Ctx& c) {
   // enough CTAs for >= 4 waves of 3 per SM (148 SMs), at most kPureRun tiles of 256^2 cells each
   // (more tiles when they are smaller: the zeroing and the flush are per run, not per cell)
   const int64_t T2 = (int64_t)c.rp.T * c.rp.T;
-  const int64_t cap = std::max<int64_t>(kPureRun, std::min<int64_t>(256, kPureRun * 65536 / std::max<int64_t>(T2, 1)));
+  const int64_t cap = std::max<int64_t>(kPureRun, std::min<int64_t>(kPureRunMax, kPureRun * 65536 / std::max<int64_t>(T2, 1)));
   const int64_t run = c.n_inside / (148 * 3 * 4);
   // the shared uint32 histogram is kept across a run of tiles: run * T^2 < 2^32 (zh_create caps T)
   const int64_t no_wrap = std::max<int64_t>(1, (int64_t)0xFFFFFFFFll / std::max<int64_t>(T2, 1));
