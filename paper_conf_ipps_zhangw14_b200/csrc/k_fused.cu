@@ -329,7 +329,7 @@ static PureP pure_params(Ctx& c) {
 template <int kMode, bool kU64>
 static void launch_pure(Ctx& c, size_t smem, unsigned grid) {
   auto k = k_fused_pure<kMode, kU64>;
-  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  prep_kernel(k, smem);
   k<<<grid, 512, smem, c.stream>>>(pure_params(c));
 }
 

@@ -399,6 +399,12 @@ cudaError_t launch_pairs_phase1(Ctx& c) {
   cudaMemsetAsync(c.d_ncand.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
   cudaMemsetAsync(c.d_nband.as<int64_t>() + P, 0, sizeof(int64_t), c.stream);
   cudaMemsetAsync(c.d_counts.p, 0, sizeof(int64_t) * 8, c.stream);
+  if (ZH_CARVEOUT >= 0) {
+    prep_kernel(k_mbb_edges, 0);
+    prep_kernel(k_poly_bands, 0);
+    prep_kernel(k_mark, 0);
+    prep_kernel(k_classify, 0);
+  }
   if (P > 0) {
     k_mbb_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
                                          c.d_y.as<double>(), c.geo, c.rp, c.d_mbb.as<int4>(), c.d_ncand.as<int64_t>(),

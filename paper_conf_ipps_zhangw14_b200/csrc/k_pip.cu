@@ -129,7 +129,7 @@ cudaError_t launch_parity(Ctx& c, const int2* pairs, int64_t grid, const int64_t
   const size_t smem = ((size_t)p.rc * p.wpr + 3) / 4 * 16;
   const bool rep = !(c.geo.ox == 0.5 && c.geo.oy == 0.5);
   void (*k)(PipP) = rep ? k_parity<true> : k_parity<false>;
-  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  prep_kernel(k, smem);
   k<<<(unsigned)grid, ZH_PAR_THREADS, smem, s>>>(p);
   c.launches += 1;
   return cudaGetLastError();
@@ -147,7 +147,7 @@ cudaError_t launch_pip_cells(Ctx& c, const int2* pairs, int64_t grid, const int6
     case 3: k = c.out_u64 ? k_pip_cells<3, true> : k_pip_cells<3, false>; break;
     default: k = c.out_u64 ? k_pip_cells<4, true> : k_pip_cells<4, false>; break;
   }
-  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  prep_kernel(k, smem);
   k<<<(unsigned)grid, kPipThreads, smem, c.stream>>>(p);
   c.launches += 1;
   return cudaGetLastError();
@@ -210,7 +210,7 @@ cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64
     default: k = ZH_MIX_K(4); break;
   }
 #undef ZH_MIX_K
-  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  prep_kernel(k, smem);
   k<<<(unsigned)grid, ZH_MIX_THREADS, smem, c.stream>>>(p);
   c.launches += 1;
   return cudaGetLastError();

@@ -36,7 +36,7 @@ __global__ void __launch_bounds__(512, 3) k_tile_hist(RasterP rp, BinP bp, FastB
 template <int kMode>
 static void launch_mode(Ctx& c, size_t smem, int threads) {
   auto k = k_tile_hist<kMode>;
-  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  prep_kernel(k, smem);
   k<<<(unsigned)c.n_tiles, threads, smem, c.stream>>>(c.rp, c.bp, make_fast_bins(c.bp), c.B_pad,
                                                       c.d_tile_hist.as<uint32_t>());
 }

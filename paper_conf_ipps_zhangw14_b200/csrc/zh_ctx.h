@@ -106,6 +106,18 @@ struct Ctx {
   int64_t graph_kernels = 0;              // kernel launches one replay performs
 };
 
+// Kernel attributes set before a launch: the dynamic shared memory beyond 48 KB it needs, and (with
+// ZH_CARVEOUT >= 0) the preferred shared-memory carveout, the same for every kernel of the step so
+// that consecutive kernels do not reconfigure the SMs' L1 / shared split.
+#ifndef ZH_CARVEOUT
+#define ZH_CARVEOUT -1
+#endif
+template <class K>
+inline void prep_kernel(K k, size_t smem) {
+  if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (ZH_CARVEOUT >= 0) cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, ZH_CARVEOUT);
+}
+
 // Timing event on stream s (an external record node while a graph is being captured).
 inline void rec_event(const Ctx& c, cudaEvent_t e, cudaStream_t s) {
   cudaEventRecordWithFlags(e, s, c.capturing ? cudaEventRecordExternal : cudaEventRecordDefault);
