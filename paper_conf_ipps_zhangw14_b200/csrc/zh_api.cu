@@ -210,8 +210,14 @@ static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bin
   for (int64_t i = 0; i < p->n_ring; ++i)
     if (p->ring_vert_off[i + 1] < p->ring_vert_off[i])
       return fail(ZH_ERR_INVALID_ARG, "ring_vert_off not non-decreasing at %lld", (long long)i);
-  // finiteness and max |coordinate| of the vertices: one pass, split over host threads for large
-  // inputs (CONUS: 9.6 M vertices, ~25 ms on one core)
+  return ZH_OK;
+}
+
+// Finiteness and max |coordinate| of the vertices (and with it the cell-size condition): one pass,
+// split over host threads for large inputs (CONUS: 9.6 M vertices, ~25 ms on one core).  zh_create
+// runs it before any CUDA call for small inputs, and for large ones while the vertex arrays are
+// already on their way to the device (the DMA hides the scan).
+static zh_status scan_vertices(const zh_raster* r, const zh_polygons* p) {
   const int64_t nv = p->n_vert;
   const int nth = nv >= (1 << 20) ? (int)std::min<unsigned>(16u, std::max(1u, std::thread::hardware_concurrency())) : 1;
   std::vector<double> part_max(nth, 0.0);
@@ -251,11 +257,34 @@ static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bin
   return ZH_OK;
 }
 
+#if defined(ZH_DESTROY_TRACE) || defined(ZH_CREATE_TRACE)
+#include <chrono>
+static double now_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+#endif
+#ifdef ZH_DESTROY_TRACE
+#define ZH_TR(label) fprintf(stderr, "zh_destroy %-10s %8.3f ms\n", label, now_ms() - t_tr), t_tr = now_ms()
+#else
+#define ZH_TR(label) (void)0
+#endif
+#ifdef ZH_CREATE_TRACE
+#define ZH_TRC(label) fprintf(stderr, "zh_create %-10s %8.3f ms\n", label, now_ms() - t_tr), t_tr = now_ms()
+#else
+#define ZH_TRC(label) (void)0
+#endif
+
 extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygons* p, const zh_bins* b,
                                const zh_options* o) {
   if (!out) return fail(ZH_ERR_INVALID_ARG, "out is NULL");
+#ifdef ZH_CREATE_TRACE
+  double t_tr = now_ms();
+#endif
   zh_status st = validate(r, p, b, o);
   if (st != ZH_OK) return st;
+  const bool scan_during_h2d = p->n_vert >= (1 << 20);
+  if (!scan_during_h2d && (st = scan_vertices(r, p)) != ZH_OK) return st;
+  ZH_TRC("validate");
   const int64_t T = o->tile;
   const int64_t TC = (r->cols + T - 1) / T;
   const int64_t tr0 = r->row0 / T;
@@ -312,6 +341,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
     return s;
   };
   cudaError_t e;
+  ZH_TRC("setup");
   // polygons: int32 offsets + coordinates, copied H2D on the stream
   std::vector<int32_t> pro(p->n_poly + 1), rvo(p->n_ring + 1);
   for (int64_t i = 0; i <= p->n_poly; ++i) pro[i] = (int32_t)p->poly_ring_off[i];
@@ -328,12 +358,14 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
         (e = cudaMemcpyAsync(c->d_y.p, p->y, (size_t)p->n_vert * 8, cudaMemcpyHostToDevice, c->stream)))
       return cleanup_fail(cuda_fail(e, "zh_create (vertices H2D)"));
   }
+  if (scan_during_h2d && (st = scan_vertices(r, p)) != ZH_OK) return cleanup_fail(st);
   // output (the per-tile histograms of step 1 are allocated by the first zh_tile_hist)
   const size_t out_bytes = (size_t)p->n_poly * b->nbins * (c->out_u64 ? 8 : 4);
   if ((e = c->d_out_own.ensure(out_bytes)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (output)"));
   c->d_out = c->d_out_own.p;
   if ((e = cudaMemsetAsync(c->d_out, 0, out_bytes, c->stream)) != cudaSuccess)
     return cleanup_fail(cuda_fail(e, "zh_create"));
+  ZH_TRC("h2d+out");
   if (c->on_host) {
     if ((e = c->raster_dev.ensure((size_t)std::max<int64_t>(r->nrows, 1) * r->pitch * 2 + 16)) != cudaSuccess)
       return cleanup_fail(cuda_fail(e, "zh_create (device raster copy)"));
@@ -354,20 +386,12 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   if ((e = cudaGetLastError()) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create"));
   // the polygon arrays are the caller's (zh.h: they may be freed or reused once zh_create
   // returns); with page-locked host arrays the copies above are truly asynchronous
+  ZH_TRC("enqueue");
   if ((e = cudaStreamSynchronize(c->stream)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (H2D)"));
+  ZH_TRC("sync");
   *out = reinterpret_cast<zh_ctx>(c);
   return ZH_OK;
 }
-
-#ifdef ZH_DESTROY_TRACE
-#include <chrono>
-static double now_ms() {
-  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
-}
-#define ZH_TR(label) fprintf(stderr, "zh_destroy %-10s %8.3f ms\n", label, now_ms() - t_tr), t_tr = now_ms()
-#else
-#define ZH_TR(label) (void)0
-#endif
 
 extern "C" void zh_destroy(zh_ctx h) {
   if (!h) return;

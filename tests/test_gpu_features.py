@@ -122,3 +122,44 @@ def test_distance_rejects_bad_ids(tiny_gpu, cuda_device):
         z.run()
         with pytest.raises(zh.ZhError):
             z.zh_hist_distance("l1", [0], [P.n_poly])
+
+
+def test_distances_with_empty_and_no_polygons(tiny_gpu, cuda_device):
+    """Polygons with no counted cell give NaN distances (R17) and NaN summaries; no polygons at all
+    give empty results."""
+    from paper_conf_ipps_zhangw14_b200 import zh
+    from synth.polygons import from_rings
+    cfg, P, R, t = tiny_gpu
+    sq = (np.array([5.0, 30, 30, 5]), np.array([5.0, 5, 30, 30]))
+    off = (sq[0] + 5000, sq[1])  # far off the raster: no cell
+    Q = from_rings([[sq], [off], [(sq[0] + 100, sq[1] + 100)]])
+    with zh.ZonalHistogram(t, cfg.gt, Q, cfg.nbins, tile=64, nodata=cfg.nodata) as z:
+        z.run()
+        M = z.zh_hist_distance("l1")
+        S = z.zh_zonal_summary()
+    assert np.isnan(M[1]).all() and np.isnan(M[:, 1]).all()
+    assert M[0, 0] == 0 and M[0, 2] == M[2, 0] and not np.isnan(M[0, 2])
+    assert S[1, 0] == 0 and np.isnan(S[1, 1:]).all()
+    E = from_rings([])
+    with zh.ZonalHistogram(t, cfg.gt, E, cfg.nbins, tile=64) as z:
+        z.run()
+        assert z.zh_hist_distance("emd").shape == (0, 0)
+        assert z.zh_zonal_summary().shape == (0, 6)
+
+
+def test_step_graph_on_host_raster(tiny_gpu, cuda_device):
+    """zh_step_graph on a context whose raster lives in host memory: after the upload (zh_run) the
+    graph replays the step on the device copy."""
+    import torch
+    from paper_conf_ipps_zhangw14_b200 import zh
+    cfg, P, R, t = tiny_gpu
+    H = oracle.o1(R, cfg.gt, P, oracle.make_bins(cfg.nbins, nodata=cfg.nodata))
+    pinned = torch.from_numpy(R.copy()).pin_memory()
+    for fused in (True, False):
+        with zh.ZonalHistogram(pinned, cfg.gt, P, cfg.nbins, tile=cfg.tile, nodata=cfg.nodata, fused=fused) as z:
+            with pytest.raises(zh.ZhError):
+                z.zh_step_graph()  # nothing uploaded yet
+            assert (z.run() == H).all()
+            for _ in range(3):
+                z.zh_step_graph()
+                assert (z.output_device().cpu().numpy().view(np.uint64) == H).all()
