@@ -1,7 +1,8 @@
-"""Simulate the N-GPU decomposition on one GPU: time each shard's step (pair_tiles + fused update)
-separately and report max / mean per N, for equal and work-balanced (zh_plan_rows) strips.
-The max over shards is the compute part of an N-GPU step (the NCCL reduce is not included).
-python tools/shard_sim.py [config]"""
+"""Simulate the N-GPU decomposition on one GPU: time each shard's step (the bench's: pair_tiles +
+fused update replayed from the context's CUDA graph, over the polygons whose bounding box meets the
+strip — dist.strip_polygons) separately and report max / mean per N, for equal and work-balanced
+(zh_plan_rows) strips.  The max over shards is the compute part of an N-GPU step (the NCCL reduce
+is not included).  python tools/shard_sim.py [config]"""
 import json
 import os
 import sys
@@ -10,7 +11,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 
 from paper_conf_ipps_zhangw14_b200 import zh  # noqa: E402
-from paper_conf_ipps_zhangw14_b200.dist import plan_shards  # noqa: E402
+from paper_conf_ipps_zhangw14_b200.dist import plan_shards, strip_polygons  # noqa: E402
 from synth.configs import CONFIGS  # noqa: E402
 from synth.dem import fill_device  # noqa: E402
 
@@ -31,15 +32,17 @@ for n in (1, 2, 4, 8):
             if b[s + 1] == b[s]:
                 times.append(0.0)
                 continue
-            with zh.ZonalHistogram(r[b[s]:b[s + 1]], cfg.gt, P, cfg.nbins, tile=cfg.tile, rows=cfg.rows,
+            Ps = P.subset(strip_polygons(P, cfg.gt, b[s], b[s + 1])) if n > 1 else P
+            with zh.ZonalHistogram(r[b[s]:b[s + 1]], cfg.gt, Ps, cfg.nbins, tile=cfg.tile, rows=cfg.rows,
                                    cols=cfg.cols, row0=b[s], nodata=cfg.nodata) as z:
                 best = 1e9
+                for _ in range(2):  # direct (learns the sizes), captured
+                    z.zh_step_graph()
                 for _ in range(3):
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                     torch.cuda.synchronize()
                     e0.record()
-                    z.zh_pair_tiles()
-                    z.zh_fused_update()
+                    z.zh_step_graph()
                     e1.record()
                     torch.cuda.synchronize()
                     best = min(best, e0.elapsed_time(e1))
