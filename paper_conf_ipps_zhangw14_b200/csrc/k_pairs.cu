@@ -18,6 +18,8 @@
 //                  at its first cell with a scanline over the band's edges (INSIDE / OUTSIDE);
 //   7. compaction— packed (inside, intersect) exclusive scan -> (tile, polygon) lists sorted by
 //                  (polygon, tile).
+#include <algorithm>
+
 #include <cub/device/device_scan.cuh>
 
 #include "zh_ctx.h"
@@ -249,19 +251,23 @@ __global__ void __launch_bounds__(256) k_mark(const int32_t* __restrict__ pro, c
   }
 }
 
-// One CTA per band (polygon k, tile row tr): classify the unmarked tiles of the row by the exact
-// PIP status of their first cell (r = tr*T, c = tc*T).  For each band edge straddling r the
-// toggled tiles {tc : xc(tc*T) < xi} form a prefix (gt1 > 0) or a suffix (gt1 < 0) of the row,
-// recorded as flips of a difference bitmap D; parity(j) = XOR_{i > j} D[i].
-__global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges, const int2* __restrict__ erows,
-                                                  const int32_t* __restrict__ band_off,
-                                                  const int32_t* __restrict__ band_edges,
-                                                  const int64_t* __restrict__ band_base,
-                                                  const int32_t* __restrict__ band_poly, Geo g, RasterP rp,
-                                                  const int4* __restrict__ mbb, const int64_t* __restrict__ cand_off,
-                                                  uint8_t* __restrict__ cls, int dwords) {
-  extern __shared__ uint32_t D[];
-  const int64_t band = blockIdx.x;
+// One WARP per band (polygon k, tile row tr; 4 bands per CTA): classify the unmarked tiles of the
+// row by the exact PIP status of their first cell (r = tr*T, c = tc*T).  For each band edge
+// straddling r the toggled tiles {tc : xc(tc*T) < xi} form a prefix (gt1 > 0) or a suffix (gt1 < 0)
+// of the row, recorded as flips of a difference bitmap D (per warp, shared memory);
+// parity(j) = XOR_{i > j} D[i].  (A band's work is a few hundred edges and a handful of tiles: a
+// warp, not a CTA, and no block-wide barrier.)
+constexpr int kClassifyWarps = 4;
+__global__ void __launch_bounds__(32 * kClassifyWarps) k_classify(
+    const Edge* __restrict__ edges, const int2* __restrict__ erows, const int32_t* __restrict__ band_off,
+    const int32_t* __restrict__ band_edges, const int64_t* __restrict__ band_base,
+    const int32_t* __restrict__ band_poly, int64_t n_bands, Geo g, RasterP rp, const int4* __restrict__ mbb,
+    const int64_t* __restrict__ cand_off, uint8_t* __restrict__ cls, int dwords) {
+  extern __shared__ uint32_t Dall[];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t band = (int64_t)blockIdx.x * (blockDim.x >> 5) + wid;
+  if (band >= n_bands) return;  // whole warps exit: only __syncwarp below
+  uint32_t* D = Dall + wid * dwords;
   const int k = band_poly[band];
   const int4 m = mbb[k];
   const int tr = m.z + (int)(band - band_base[k]);
@@ -269,10 +275,11 @@ __global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges
   const int64_t rrep = (int64_t)tr * rp.T;
   const double yc = row_centre(g, rrep);
   const bool s = g.gt1 > 0;
-  for (int i = threadIdx.x; i < dwords; i += blockDim.x) D[i] = 0;
-  __syncthreads();
+  const int nd = (wk >> 5) + 1;
+  for (int i = lane; i < nd; i += 32) D[i] = 0;
+  __syncwarp();
   const int e0 = band_off[band], e1 = band_off[band + 1];
-  for (int i = e0 + threadIdx.x; i < e1; i += blockDim.x) {
+  for (int i = e0 + lane; i < e1; i += 32) {
     const int v = band_edges[i];
     const int2 rr = erows[v];
     if (!(rr.x <= rrep && rrep < rr.y)) continue;
@@ -286,8 +293,8 @@ __global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges
     if (jb > 0) atomicXor(&D[jb >> 5], 1u << (jb & 31));
     if (!s) atomicXor(&D[wk >> 5], 1u << (wk & 31));
   }
-  __syncthreads();
-  if (threadIdx.x == 0) {
+  __syncwarp();
+  if (lane == 0) {
     uint32_t carry = 0;
     for (int wi = (wk >> 5); wi >= 0; --wi) {
       uint32_t t = D[wi];
@@ -296,9 +303,9 @@ __global__ void __launch_bounds__(128) k_classify(const Edge* __restrict__ edges
       carry ^= (t & 1u);
     }
   }
-  __syncthreads();
+  __syncwarp();
   uint8_t* c = cls + cand_off[k] + (int64_t)(tr - m.z) * wk;
-  for (int j = threadIdx.x; j < wk; j += blockDim.x) {
+  for (int j = lane; j < wk; j += 32) {
     if (c[j] == 0) c[j] = ((D[j >> 5] >> (j & 31)) & 1u) ? 1 : 3;
   }
 }
@@ -465,11 +472,14 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
         c.launches += 1;
       }
       const int dwords = c.rp.TC / 32 + 2;
-      k_classify<<<(unsigned)nb, 128, sizeof(uint32_t) * dwords, c.stream>>>(
+      // warps (bands) per CTA: 4, fewer when a band's bitmap is large (TC <= 2^20: zh_create)
+      const int nw = (int)std::max<int64_t>(1, std::min<int64_t>(kClassifyWarps, 48 * 1024 / (4 * dwords)));
+      const size_t smem = sizeof(uint32_t) * (size_t)dwords * nw;
+      prep_kernel(k_classify, smem);
+      k_classify<<<(unsigned)((nb + nw - 1) / nw), 32 * nw, smem, c.stream>>>(
           c.d_edges.as<Edge>(), c.d_erows.as<int2>(), c.d_band_off.as<int32_t>(), c.d_band_edges.as<int32_t>(),
-          c.d_band_base.as<int64_t>(), c.d_band_poly.as<int32_t>(), c.geo, c.rp, c.d_mbb.as<int4>(),
-          c.d_cand_off.as<int64_t>(),
-          c.d_class.as<uint8_t>(), dwords);
+          c.d_band_base.as<int64_t>(), c.d_band_poly.as<int32_t>(), nb, c.geo, c.rp, c.d_mbb.as<int4>(),
+          c.d_cand_off.as<int64_t>(), c.d_class.as<uint8_t>(), dwords);
       c.launches += 1;
     }
     k_flags<<<grid_for(nc, 256), 256, 0, c.stream>>>(c.d_class.as<uint8_t>(), nc, c.d_flags.as<uint64_t>());

@@ -291,6 +291,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   const int64_t TRn = (r->nrows + T - 1) / T;
   const int64_t n_tiles = TC * TRn;
   if (n_tiles >= (1ll << 31) || TC >= (1ll << 31)) return fail(ZH_ERR_UNSUPPORTED, "more than 2^31 tiles");
+  if (TC > (1ll << 20)) return fail(ZH_ERR_UNSUPPORTED, "more than 2^20 tile columns (step 2's row bitmaps)");
   if (!o->out_u64) {
     // uint32 output: a polygon's count is bounded by the cells of its MBB
     for (int64_t k = 0; k < p->n_poly; ++k) {
