@@ -386,11 +386,13 @@ def main():
     kern = {}
     if path == "fused":
         kern["k_fused_pure"] = (avg(lib_ms, "fused_pure_kernel"), 2.0 * st["n_pure_cells"])
-        # mixed tiles: k_mixed_cells reads a tile once per group of <= 2 pairs (n_group_cells); the
-        # per-pair k_pip_cells (when the grouped form does not apply) once per pair
-        cell_k = "k_mixed_cells" if st["n_mixed_groups"] > 0 else "k_pip_cells"
-        kern[cell_k] = (avg(lib_ms, "fused_pip_kernel"),
-                        2.0 * (st["n_group_cells"] if st["n_mixed_groups"] > 0 else st["n_pip_cells"]))
+        # mixed tiles: the HBM bytes k_mixed_cells must read are every mixed tile's cells once
+        # (n_mixed_cells; a tile's later groups of <= 2 pairs re-read it from L2 — n_group_cells
+        # counts those too and is reported beside); the per-pair k_pip_cells (when the grouped form
+        # does not apply) reads a tile once per pair
+        grouped = st["n_mixed_groups"] > 0
+        cell_k = "k_mixed_cells" if grouped else "k_pip_cells"
+        kern[cell_k] = (avg(lib_ms, "fused_pip_kernel"), 2.0 * (st["n_mixed_cells"] if grouped else st["n_pip_cells"]))
         steps_detail = {"step2_pair_tiles": {"ms": avg(lib_ms, "step2_pair_tiles")},
                         "fused_update(steps1+3+4)": {"ms": avg(lib_ms, "fused_update")}}
     else:
@@ -401,6 +403,10 @@ def main():
         steps_detail = {"step2_pair_tiles": {"ms": avg(lib_ms, "step2_pair_tiles")}}
     for name, (t, b) in kern.items():
         steps_detail[name] = {"ms": t, "alg_bytes": b, "alg_GBps": b / (t / 1000.0) / 1e9 if t else None}
+    if path == "fused" and st["n_mixed_groups"] > 0:
+        t = steps_detail["k_mixed_cells"]["ms"]
+        steps_detail["k_mixed_cells"]["group_read_bytes"] = 2.0 * st["n_group_cells"]  # incl. L2 re-reads
+        steps_detail["k_mixed_cells"]["group_read_GBps"] = 2.0 * st["n_group_cells"] / (t / 1000.0) / 1e9 if t else None
     if path == "fused":
         # the parity bitmaps of the mixed pairs (FP64 crossing work; after k_fused_pure, exact grid)
         steps_detail["k_parity"] = {"ms": avg(lib_ms, "fused_parity_kernel")}

@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define ZH_ABI_VERSION 7
+#define ZH_ABI_VERSION 8
 
 typedef struct zh_ctx_s* zh_ctx;
 
@@ -151,6 +151,8 @@ typedef struct {
   int64_t n_mixed_groups; /* after zh_fused_update: tile groups (<= 2 pairs of one tile) of the
                              grouped cell kernel (0 when it does not apply)                      */
   int64_t n_group_cells;  /* cells those groups read (a mixed tile once per group)              */
+  int64_t n_mixed_cells;  /* cells of the mixed tiles, each once (the HBM bytes the grouped cell
+                             kernel must read: a tile's later groups find it in L2)              */
 } zh_stats;
 
 /* Validate, copy polygons to the device (H2D on options->stream), allocate per-tile histograms

@@ -132,21 +132,28 @@ __global__ void k_pack_mixed(const uint32_t* __restrict__ cnt, int64_t n, uint64
 
 
 // grp[g] = {first pair index, #pairs}; counts[4] = #groups, counts[5] = cells read by the groups
-// (a mixed tile once per group: the grouped cell kernel's algorithmic bytes)
+// (a mixed tile once per group), counts[6] = cells of the mixed tiles (each once: the HBM bytes the
+// grouped cell kernel must read — later groups of a tile find it in L2)
 __global__ void k_pip_groups(const uint32_t* __restrict__ cnt, const uint64_t* __restrict__ off, int64_t n_tiles,
                              RasterP rp, int2* __restrict__ grp, int64_t* __restrict__ counts) {
-  int64_t cells = 0;
+  int64_t cells = 0, tcells = 0;
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n_tiles; t += (int64_t)gridDim.x * blockDim.x) {
     const uint32_t c = cnt[t];
     if (!c) continue;
     const uint32_t p0 = (uint32_t)off[t], g0 = (uint32_t)(off[t] >> 32);
     for (uint32_t q = 0; 2 * q < c; ++q) grp[g0 + q] = make_int2((int)(p0 + 2 * q), (int)min(2u, c - 2 * q));
     cells += tile_cells(rp, (int)t) * (int64_t)((c + 1) >> 1);
+    tcells += tile_cells(rp, (int)t);
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) counts[4] = (int64_t)(off[n_tiles] >> 32);
-  for (int o = 16; o > 0; o >>= 1) cells += __shfl_xor_sync(0xffffffffu, cells, o);
-  if ((threadIdx.x & 31) == 0 && cells) atomicAdd(reinterpret_cast<unsigned long long*>(&counts[5]),
-                                                  (unsigned long long)cells);
+  for (int o = 16; o > 0; o >>= 1) {
+    cells += __shfl_xor_sync(0xffffffffu, cells, o);
+    tcells += __shfl_xor_sync(0xffffffffu, tcells, o);
+  }
+  if ((threadIdx.x & 31) == 0 && cells) {
+    atomicAdd(reinterpret_cast<unsigned long long*>(&counts[5]), (unsigned long long)cells);
+    atomicAdd(reinterpret_cast<unsigned long long*>(&counts[6]), (unsigned long long)tcells);
+  }
 }
 
 struct PureP {
@@ -361,9 +368,9 @@ cudaError_t launch_fused(Ctx& c) {
   if ((e = c.d_extra_pos.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_mixed_pk.ensure(sizeof(uint64_t) * ((size_t)NT + 1))) != cudaSuccess) return e;
   if ((e = c.d_pip.ensure(sizeof(int2) * ((size_t)NI + NX + 1))) != cudaSuccess) return e;
-  if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 6)) != cudaSuccess) return e;
+  if ((e = c.d_fcounts.ensure(sizeof(int64_t) * 7)) != cudaSuccess) return e;
   if (c.cover && (e = c.d_remap.ensure(sizeof(int32_t) * ((size_t)NX + 1))) != cudaSuccess) return e;
-  cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 6, c.stream);
+  cudaMemsetAsync(c.d_fcounts.p, 0, sizeof(int64_t) * 7, c.stream);
   if (NT == 0 || NI + NX == 0) {
     if (c.timing)
       for (int i = 10; i < 16; ++i) rec_event(c, c.ev[i], c.stream);

@@ -922,10 +922,11 @@ extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
   s->device_bytes = (int64_t)zh::device_bytes(*c);
   s->h2d_bytes = c->h2d_bytes;
   s->n_pure_tiles = s->n_pip_pairs = s->n_pure_cells = s->n_pip_cells = s->n_mixed_groups = s->n_group_cells = 0;
+  s->n_mixed_cells = 0;
   zh_status fs = check_flag(c, "zh_get_stats");
   if (fs != ZH_OK) return fs;
   if (c->fused_done) {
-    ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_fcounts.p, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
+    ZH_CU(cudaMemcpyAsync(c->pinned_counts, c->d_fcounts.p, 7 * sizeof(int64_t), cudaMemcpyDeviceToHost, c->stream),
           "zh_get_stats");
     ZH_CU(cudaStreamSynchronize(c->stream), "zh_get_stats");
     s->n_pure_tiles = c->pinned_counts[0];
@@ -934,6 +935,7 @@ extern "C" zh_status zh_get_stats(zh_ctx h, zh_stats* s) {
     s->n_pip_cells = c->pinned_counts[3];
     s->n_mixed_groups = c->pinned_counts[4];
     s->n_group_cells = c->pinned_counts[5];
+    s->n_mixed_cells = c->pinned_counts[6];
   }
   return ZH_OK;
 }

@@ -62,7 +62,8 @@ class zh_stats(ctypes.Structure):
                 ("n_isect", ctypes.c_int64), ("n_band_entries", ctypes.c_int64), ("n_edges", ctypes.c_int64),
                 ("device_bytes", ctypes.c_int64), ("n_pure_tiles", ctypes.c_int64), ("n_pip_pairs", ctypes.c_int64),
                 ("n_pure_cells", ctypes.c_int64), ("n_pip_cells", ctypes.c_int64), ("h2d_bytes", ctypes.c_int64),
-                ("n_mixed_groups", ctypes.c_int64), ("n_group_cells", ctypes.c_int64)]
+                ("n_mixed_groups", ctypes.c_int64), ("n_group_cells", ctypes.c_int64),
+                ("n_mixed_cells", ctypes.c_int64)]
 
 
 EXPORTS = ["zh_create", "zh_upload_raster", "zh_tile_hist", "zh_pair_tiles", "zh_aggregate", "zh_pip_update",

@@ -33,7 +33,7 @@ def test_library_exports_every_declared_symbol():
     assert not missing, missing
     from paper_conf_ipps_zhangw14_b200 import zh
     assert set(zh.EXPORTS) == set(_declared())
-    assert zh.LIB.zh_abi_version() == 7
+    assert zh.LIB.zh_abi_version() == 8
 
 
 def test_library_is_sm100a_sass():
