@@ -541,7 +541,8 @@ extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect
     // the sizes are those of the first call (fixed geometry): no host round trip; the device
     // checks the recomputed counts against them
     ZH_CU(zh::launch_pairs_phase2(*c), "zh_pair_tiles (phase 2)");
-    const int64_t want[6] = {c->n_cand, c->n_bands, c->n_band_entries, 0, c->n_inside, c->n_isect};
+    const int64_t want[6] = {c->n_cand + c->n_cand_check_bias, c->n_bands, c->n_band_entries, 0, c->n_inside,
+                             c->n_isect};
     ZH_CU(zh::launch_check_counts(*c, c->d_counts.as<int64_t>(), want, 3), "zh_pair_tiles (check)");
     ZH_CU(zh::launch_check_counts(*c, c->d_counts.as<int64_t>() + 4, want + 4, 2), "zh_pair_tiles (check)");
     toc(c, 1);
@@ -564,6 +565,14 @@ extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect
     c->n_inside = c->pinned_counts[4];
     c->n_isect = c->pinned_counts[5];
     c->sizes_known = true;
+    // ZH_TEST_BAD_SIZES=1 (testing the guard): remember a wrong candidate count, so that the next
+    // host-sync-free step's device check must flag it
+    const char* bad = getenv("ZH_TEST_BAD_SIZES");
+    if (bad && bad[0] == '1') c->bad_sizes_pending = true;
+  }
+  if (c->bad_sizes_pending && c->sizes_known) {
+    c->bad_sizes_pending = false;
+    c->n_cand_check_bias = 1;
   }
   c->have_pairs = true;
   if (n_inside) *n_inside = c->n_inside;

@@ -104,6 +104,8 @@ struct Ctx {
   cudaGraphExec_t gexec = nullptr;
   int32_t graph_fused = -1;               // the path the graph was captured for
   int64_t graph_kernels = 0;              // kernel launches one replay performs
+  bool bad_sizes_pending = false;         // ZH_TEST_BAD_SIZES: test hook of the device size check
+  int64_t n_cand_check_bias = 0;
 };
 
 // Kernel attributes set before a launch: the dynamic shared memory beyond 48 KB it needs, and (with

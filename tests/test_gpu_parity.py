@@ -454,3 +454,28 @@ def test_step_graph_replays(tiny, cuda_device, fused):
             assert (out2.cpu().numpy().view(np.uint64) == H).all(), i
         st = z.stats()  # a syncing call: also checks the device count guard
         assert st["n_isect"] > 0
+
+
+def test_known_sizes_guard_fires(tiny, cuda_device, monkeypatch):
+    """The host-sync-free steps trust the list sizes learnt by a context's first zh_pair_tiles; the
+    device check must report a step whose counts differ (ZH_TEST_BAD_SIZES makes the context
+    remember a wrong candidate count): the next syncing call fails with ZH_ERR_STATE."""
+    zh = _zh()
+    cfg, P, R, H = tiny
+    t = device_raster(cfg.dem, cfg.rows, cfg.cols)
+    monkeypatch.setenv("ZH_TEST_BAD_SIZES", "1")
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=cfg.tile, cols=cfg.cols, nodata=cfg.nodata) as z:
+        z.zh_pair_tiles()      # learns the sizes (and, under the hook, a wrong candidate count)
+        z.zh_fused_update()
+        z.zh_pair_tiles()      # host-sync-free: the device check compares
+        z.zh_fused_update()
+        with pytest.raises(zh.ZhError) as ei:
+            z.stats()
+        assert ei.value.status == zh.ZH_ERR_STATE
+    monkeypatch.delenv("ZH_TEST_BAD_SIZES")
+    with zh.ZonalHistogram(t, cfg.gt, P, cfg.nbins, tile=cfg.tile, cols=cfg.cols, nodata=cfg.nodata) as z:
+        for _ in range(3):
+            z.zh_pair_tiles()
+            z.zh_fused_update()
+        z.stats()  # no mismatch: no error
+        assert (z.output_device().cpu().numpy().view(np.uint64) == H).all()
