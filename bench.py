@@ -96,6 +96,23 @@ METRIC = ("raster cells/s (zonal histogram of the whole raster; device step = pa
           "with raster and polygons resident in HBM; e2e objects: host-side end to end)")
 
 
+def host_info() -> dict:
+    """The host the CPU oracle runs on (record nproc, the CPU model and host DRAM)."""
+    model, mem = None, None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal"):
+                mem = round(int(line.split()[1]) / 2 ** 20, 1)
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model, "host_mem_gib": mem}
+
+
 def measured_peaks() -> dict:
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -188,7 +205,8 @@ def run_reference(args, cfg):
             "unit": "cells/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "i16",
             "data": "synthetic", "config": cfg.describe(),
-            "cpu_baseline": {"value": value, "unit": "cells/s", "cores": threads, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "cells/s", "cores": threads, "kind": "oracle", "sample": sample,
+                             "host": host_info()},
             "e2e": {"value": value, "unit": "cells/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -480,7 +498,7 @@ def main():
         else:
             band = raster_v[start:start + n, :cfg.cols].cpu().numpy()
         dt, cnt, threads = oracle_band(cfg, P, start, n, host_rows=band)
-        cpu = {"value": n * cfg.cols / dt, "unit": "cells/s", "cores": threads, "kind": "oracle",
+        cpu = {"value": n * cfg.cols / dt, "unit": "cells/s", "cores": threads, "kind": "oracle", "host": host_info(),
                "sample": f"rows [{start},{start + n}) x all {cfg.cols} cols of {cfg.name} ({n * cfg.cols} cells, "
                          f"{P.n_poly} polygons), oracle O1 on {threads} host threads, {dt:.1f} s"}
 
