@@ -19,6 +19,22 @@
 
 using zh::Ctx;
 
+// NVTX ranges around the ABI calls (header-only NVTX 3: free when no tool is attached), so nsys /
+// ncu timelines show the paper's steps by name.
+#ifndef ZH_NVTX
+#define ZH_NVTX 1
+#endif
+#if ZH_NVTX
+#include <nvtx3/nvToolsExt.h>
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+#define ZH_RANGE(name) NvtxRange zh_nvtx_range_(name)
+#else
+#define ZH_RANGE(name) (void)0
+#endif
+
 static thread_local char g_err[512] = "";
 
 static zh_status fail(zh_status s, const char* fmt, ...) {
@@ -276,6 +292,7 @@ static double now_ms() {
 
 extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygons* p, const zh_bins* b,
                                const zh_options* o) {
+  ZH_RANGE("zh_create");
   if (!out) return fail(ZH_ERR_INVALID_ARG, "out is NULL");
 #ifdef ZH_CREATE_TRACE
   double t_tr = now_ms();
@@ -464,6 +481,7 @@ static zh_status check_flag(Ctx* c, const char* who) {
 }
 
 extern "C" zh_status zh_upload_raster(zh_ctx h) {
+  ZH_RANGE("zh_upload_raster");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (!c->on_host) return ZH_OK;
@@ -516,6 +534,7 @@ static zh_status upload_needed(Ctx* c) {
 }
 
 extern "C" zh_status zh_tile_hist(zh_ctx h) {
+  ZH_RANGE("zh_tile_hist");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   ZH_CU(c->d_tile_hist.ensure((size_t)c->n_tiles * c->B_pad * 4), "zh_tile_hist (allocating tile histograms)");
@@ -527,6 +546,7 @@ extern "C" zh_status zh_tile_hist(zh_ctx h) {
 }
 
 extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect) {
+  ZH_RANGE("zh_pair_tiles");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   c->have_pairs = false;
@@ -581,6 +601,7 @@ extern "C" zh_status zh_pair_tiles(zh_ctx h, int64_t* n_inside, int64_t* n_isect
 }
 
 extern "C" zh_status zh_aggregate(zh_ctx h) {
+  ZH_RANGE("zh_aggregate");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (!c->have_pairs || !c->have_hist) return fail(ZH_ERR_STATE, "zh_aggregate needs zh_tile_hist and zh_pair_tiles");
@@ -594,6 +615,7 @@ extern "C" zh_status zh_aggregate(zh_ctx h) {
 }
 
 extern "C" zh_status zh_pip_update(zh_ctx h) {
+  ZH_RANGE("zh_pip_update");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (!c->have_pairs) return fail(ZH_ERR_STATE, "zh_pip_update needs zh_pair_tiles");
@@ -607,6 +629,7 @@ extern "C" zh_status zh_pip_update(zh_ctx h) {
 }
 
 extern "C" zh_status zh_fused_update(zh_ctx h) {
+  ZH_RANGE("zh_fused_update");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (!c->have_pairs) return fail(ZH_ERR_STATE, "zh_fused_update needs zh_pair_tiles");
@@ -620,6 +643,7 @@ extern "C" zh_status zh_fused_update(zh_ctx h) {
 }
 
 extern "C" zh_status zh_run(zh_ctx h, void* host_out) {
+  ZH_RANGE("zh_run");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   zh_status s;
@@ -657,6 +681,7 @@ static zh_status run_step_calls(zh_ctx h) {
 }
 
 extern "C" zh_status zh_step_graph(zh_ctx h) {
+  ZH_RANGE("zh_step_graph");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (c->on_host && c->rp.nrows > 0 && c->h2d_bytes == 0)
@@ -712,6 +737,7 @@ extern "C" zh_status zh_step_graph(zh_ctx h) {
 }
 
 extern "C" zh_status zh_zonal_stats(zh_ctx h, int64_t* host_stats, int64_t** dptr) {
+  ZH_RANGE("zh_zonal_stats");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   if (!c->have_pairs || !(c->fused_done || (c->step3_done && c->step4_done)))
@@ -738,6 +764,7 @@ static zh_status stats_on_device(Ctx* c, const char* who) {
 }
 
 extern "C" zh_status zh_zonal_summary(zh_ctx h, double* host_out, double** dptr) {
+  ZH_RANGE("zh_zonal_summary");
   if (!h) return fail(ZH_ERR_INVALID_ARG, "null context");
   Ctx* c = C(h);
   zh_status s = stats_on_device(c, "zh_zonal_summary");
@@ -756,6 +783,7 @@ extern "C" zh_status zh_zonal_summary(zh_ctx h, double* host_out, double** dptr)
 
 extern "C" zh_status zh_hist_distance(zh_ctx h, int32_t kind, const int32_t* a_ids, const int32_t* b_ids, int64_t n,
                                       double* host_out) {
+  ZH_RANGE("zh_hist_distance");
   if (!h || !host_out) return fail(ZH_ERR_INVALID_ARG, "null argument");
   Ctx* c = C(h);
   if (kind != ZH_DIST_L1 && kind != ZH_DIST_EMD && kind != ZH_DIST_CHI2)
@@ -809,6 +837,7 @@ extern "C" zh_status zh_hist_distance(zh_ctx h, int32_t kind, const int32_t* a_i
 
 extern "C" zh_status zh_plan_rows(const zh_raster* r, const zh_polygons* p, const zh_options* o, int32_t n_shards,
                                   int64_t* row_bounds, double* shard_cost) {
+  ZH_RANGE("zh_plan_rows");
   if (!r || !p || !o || !row_bounds) return fail(ZH_ERR_INVALID_ARG, "null argument");
   if (n_shards < 1) return fail(ZH_ERR_INVALID_ARG, "n_shards must be >= 1");
   // Geometry only: the raster values are never read by step 2, so a placeholder pointer stands in
