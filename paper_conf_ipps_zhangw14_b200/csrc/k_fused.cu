@@ -94,7 +94,7 @@ __global__ void k_pure_tiles(const uint32_t* __restrict__ pure_cnt, int64_t n, c
 // counts[1] = #pairs for the cell-in-polygon kernel, counts[3] = their tiles' cells.  The list is
 // grouped BY TILE (pip_off = exclusive scan of pip_cnt), so the 2-3 pairs that read the same mixed
 // tile run back to back and all but the first find its cells in L2 (grouped by polygon, as step 2
-// emits them, the L2 hit rate of k_pip was 15 %).
+// emits them, the L2 hit rate of the per-pair cell pass was 15 %).
 __global__ void k_pip_list(const int2* __restrict__ isect, int64_t n_isect, const int2* __restrict__ inside,
                            int64_t n_inside, const uint32_t* __restrict__ extra, const uint64_t* __restrict__ pip_off,
                            uint32_t* __restrict__ cursor, int64_t n_tiles, RasterP rp, int2* __restrict__ pip,

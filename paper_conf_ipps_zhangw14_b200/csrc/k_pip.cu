@@ -6,15 +6,16 @@
 //
 // Paper design (prior art): one block per polygon, one thread per cell, and for every cell a loop
 // over ALL polygon vertices in global memory with float coordinates; the histogram update is a
-// non-atomic read-modify-write (a race).  B200 design, bit-identical to the per-cell test:
+// non-atomic read-modify-write (a race).  B200 design, bit-identical to the per-cell test, in two
+// kernels (k_parity, then k_pip_cells for the four-step path or k_mixed_cells for the fused one):
 //   * one CTA per intersecting pair; only the edges of the pair's band (edges that straddle one
 //     of the tile's centre rows, built in step 2) are visited;
 //   * the crossing test `xc < xi` depends on the cell only through xc, and xc is monotone in the
 //     column, so for each (edge, row) the crossed cells form a prefix (gt1 > 0) or suffix
 //     (gt1 < 0) of the row: the exact boundary column is found with the SAME xc(c) expression
 //     (first_false), and recorded as a flip in a per-row difference bitmap in shared memory;
-//     a suffix-XOR turns it into the per-cell parity (inside) bits.  Work per pair is
-//     O(#(edge,row) crossings + cells) instead of O(cells x edges);
+//     a suffix-XOR turns it into the per-cell parity (inside) bits, stored as the pair's bitmap
+//     (k_parity).  Work per pair is O(#(edge,row) crossings + cells) instead of O(cells x edges);
 //   * edges entirely left / right of the tile's centres (with half a cell of margin, far above
 //     the intercept's rounding) skip the division;
 //   * the cells are then streamed exactly like step 1 (16-byte vectors, packed 16x2 bin mapping,

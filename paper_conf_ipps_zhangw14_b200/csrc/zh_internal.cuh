@@ -24,7 +24,7 @@ struct Geo {
 };
 
 // kRep = false: the centre (0.5 as an immediate — the hot kernels are instantiated for it, the
-// runtime offsets cost ~12 % in k_pip); kRep = true: the runtime offsets g.ox, g.oy.  Both give
+// runtime offsets cost ~12 % in the round-1 one-kernel step 4); kRep = true: the runtime offsets g.ox, g.oy.  Both give
 // identical values when the offsets are 0.5.
 template <bool kRep = true>
 __device__ __forceinline__ double col_centre(const Geo& g, int64_t c) {

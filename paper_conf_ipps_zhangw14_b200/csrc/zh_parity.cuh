@@ -1,5 +1,4 @@
-// zh_parity.cuh — the per-(tile, polygon) inside mask of step 4, shared by k_pip (one pair per CTA)
-// and k_fused_mixed (all pairs of a tile per CTA).
+// zh_parity.cuh — the per-(tile, polygon) inside mask of step 4 (k_parity, one pair per CTA).
 //
 // For a chunk of the tile's rows [rlo, rhi) and columns [c0, c0 + w), the ray-crossing parity of
 // every cell centre (Fig. 5, canonical orientation R8, half-open rule R10) is built as

@@ -54,7 +54,7 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev);  // k_pip.cu
 // ------------------------------------------------------------------------------------------------
 
 // Parity bits of pair `pair_idx` into p.pbits[pair_idx][r][0..wpo) (rows r < h of the tile).
-// `bm` holds rc * wpr words; `lq` as for pip_pair_body.
+// `bm` holds rc * wpr words; `lq` (LongQ, zh_parity.cuh) is the CTA's long-edge queue.
 template <bool kRep>
 __device__ __forceinline__ void parity_pair_body(const PipP& p, int64_t pair_idx, uint32_t* __restrict__ bm,
                                                  LongQ* lq) {
