@@ -479,3 +479,75 @@ def test_known_sizes_guard_fires(tiny, cuda_device, monkeypatch):
             z.zh_fused_update()
         z.stats()  # no mismatch: no error
         assert (z.output_device().cpu().numpy().view(np.uint64) == H).all()
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_configurations_fuzz(cuda_device, seed):
+    """Seeded random configurations against the literal O0: raster size and pitch, geotransform
+    (dyadic or lon/lat, either orientation), tile size, bin mapping (lo, width, nbins, clamp / drop,
+    nodata in or below the range), output width, and random polygons (stars, boxes on centres,
+    holes, overlaps, degenerate rings) — both libzh paths and the CUDA-graph step."""
+    import torch
+    zh = _zh()
+    rng = np.random.default_rng(1000 + seed)
+    rows, cols = int(rng.integers(40, 300)), int(rng.integers(40, 300))
+    pitch = (cols + 7) // 8 * 8 + 8 * int(rng.integers(0, 3))
+    if rng.random() < 0.5:
+        cs = 1.0 / 3600.0
+        gt = [-100.0, cs, 0.0, 40.0, 0.0, -cs]
+    else:
+        cs = float(rng.choice([0.5, 1.0, 2.0]))
+        gt = [0.0, cs, 0.0, rows * cs, 0.0, -cs]
+    if rng.random() < 0.3:  # mirrored x
+        gt[0], gt[1] = gt[0] + cols * gt[1], -gt[1]
+    if rng.random() < 0.3:  # mirrored y
+        gt[3], gt[5] = gt[3] + rows * gt[5], -gt[5]
+    tile = int(rng.choice([1, 3, 8, 16, 17, 32, 64, 100, 128, 256]))
+    spec = DemSpec(seed=int(rng.integers(1, 1000)), base=-150, macro_amp=900, fine_amp=200,
+                   void_thresh=int(rng.choice([12500, 30000])))
+    lo = int(rng.integers(-200, 100))
+    width = int(rng.choice([1, 1, 2, 7]))
+    nbins = int(rng.integers(1, 600))
+    drop = bool(rng.random() < 0.3)
+    nodata = [None, -32768, int(rng.integers(-200, 300))][int(rng.integers(0, 3))]
+    out_u64 = bool(rng.random() < 0.7)
+    X = lambda c: gt[0] + c * gt[1]
+    Y = lambda r: gt[3] + r * gt[5]
+    polys = []
+    for _ in range(int(rng.integers(1, 9))):
+        kind = rng.random()
+        if kind < 0.6:  # jagged star
+            cr, cc = rng.uniform(0, rows), rng.uniform(0, cols)
+            n = int(rng.integers(3, 60))
+            th = np.sort(rng.uniform(0, 2 * np.pi, n))
+            rad = rng.uniform(2, max(rows, cols) / 2, n)
+            rr, ccs = cr + rad * np.sin(th), cc + rad * np.cos(th)
+            if rng.random() < 0.3:  # some vertices exactly on centres
+                rr, ccs = np.floor(rr) + 0.5, np.floor(ccs) + 0.5
+            ring = (X(ccs), Y(rr))
+            rings = [ring]
+            if rng.random() < 0.3:  # a hole
+                rings.append((X(cc + 0.3 * (ccs - cc)), Y(cr + 0.3 * (rr - cr))))
+            polys.append(rings)
+        elif kind < 0.85:  # box with corners on grid lines or centres
+            r0, c0 = rng.integers(-5, rows), rng.integers(-5, cols)
+            h, w = rng.integers(1, rows), rng.integers(1, cols)
+            off = float(rng.choice([0.0, 0.5]))
+            xs = X(np.array([c0, c0 + w, c0 + w, c0]) + off)
+            ys = Y(np.array([r0, r0, r0 + h, r0 + h]) + off)
+            polys.append([(xs, ys)])
+        else:  # degenerate
+            polys.append([(X(np.array([1.0, 5.0])), Y(np.array([1.0, 5.0])))])
+    P = from_rings(polys)
+    R = fill_host(spec, cols, 0, 0, rows, cols)
+    H = oracle.o0(R, gt, P, oracle.make_bins(nbins, lo=lo, width=width, nodata=nodata, oor_drop=drop))
+    t = device_raster(spec, rows, cols, pitch=pitch)
+    kw = dict(lo=lo, width=width, nodata=nodata, oor_drop=drop, out_u64=out_u64)
+    G = gpu_hist(t, gt, P, nbins, tile, cols, **kw)
+    assert (G.astype(np.uint64) == H).all(), (seed, tile, lo, width, nbins, drop, nodata)
+    with zh.ZonalHistogram(t, gt, P, nbins, tile=tile, cols=cols, **kw) as z:
+        for _ in range(3):
+            z.zh_step_graph()
+        got = z.output_device().cpu().numpy()
+    got = got.view(np.uint64) if out_u64 else got.view(np.uint32)
+    assert (got.astype(np.uint64) == H).all(), seed
