@@ -133,7 +133,13 @@ struct FastBins {
   uint32_t L2, H2, C2, nod2;   // plain
   uint32_t Hb2, Nb2, Lb2, Cb2;  // biased
   uint32_t use_nodata, bias;
+  uint32_t nC2, nNb2, nCb2;     // -C2, -Nb2, -Cb2 per half: the kernels add them (VIADD.16x2 of a
+                                // kernel parameter, no per-use negation)
 };
+
+#ifndef ZH_NEG
+#define ZH_NEG 1
+#endif
 
 __host__ __device__ inline bool fast_bins_ok(const BinP& b) {
   return b.width == 1 && b.lo >= -32768 && b.lo <= 32767 && b.nbins <= 16000;
@@ -163,23 +169,28 @@ __host__ __device__ inline FastBins make_fast_bins(const BinP& b) {
   f.Nb2 = pk(N1);
   f.Lb2 = pk(L - N1);
   f.Cb2 = pk(C - N1);
+  f.nC2 = pk(-C);
+  f.nNb2 = pk(-N1);
+  f.nCb2 = pk(N1 - C);
   const int nod_idx = 0xFFFF - ((C - N1) & 0xFFFF);  // where a nodata cell lands
   f.bias = (b.use_nodata && b.nodata < L && (b.drop || b.nodata == -32768) && nod_idx >= hist_dummy(b.nbins) + 32)
                ? 1u : 0u;
   return f;
 }
 
-template <int kForm>  // 0 plain, 1 plain + nodata zero-detect, 2 biased (nodata below range)
+// kNeg: add the pre-negated constants (k_mixed_cells: fewer operations per vector; the pure-tile
+// kernel is slower with them, 3.16 -> 3.43 ms at CONUS — its register allocation changes)
+template <int kForm, bool kNeg = false>  // 0 plain, 1 plain + nodata zero-detect, 2 biased (nodata below range)
 __device__ __forceinline__ uint32_t fast_idx2(uint32_t w, const FastBins& f) {
   if (kForm == 2) {
     uint32_t a = __vmins2(w, f.Hb2);
-    a = __vsub2(a, f.Nb2);
+    a = kNeg ? __vadd2(a, f.nNb2) : __vsub2(a, f.Nb2);
     a = __vmaxu2(a, f.Lb2);
-    return __vsub2(a, f.Cb2);
+    return kNeg ? __vadd2(a, f.nCb2) : __vsub2(a, f.Cb2);
   }
   uint32_t c = __vmaxs2(w, f.L2);
   c = __vmins2(c, f.H2);
-  c = __vsub2(c, f.C2);
+  c = kNeg ? __vadd2(c, f.nC2) : __vsub2(c, f.C2);
   if (kForm == 1) {
     const uint32_t x = w ^ f.nod2;                 // zero halves where v == nodata
     const uint32_t z = __vsub2(x, 0x00010001u) & ~x & 0x80008000u;
@@ -259,6 +270,31 @@ __device__ __forceinline__ void count8_fast_code(uint32_t* __restrict__ hist, co
     const uint32_t j = (uint32_t)(i & 1) * 2;  // first of the two cells within its 4-cell code word
     const uint32_t P = 4u | (j << 4) | (4u << 8) | ((j + 1) << 12);
     uint32_t x = fast_idx2<kForm>(ws[i], f) | __byte_perm(i < 2 ? clo : chi, 0u, P);
+    x = __vminu2(x, dumB2) << 2;
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);
+  }
+}
+
+// count8_fast_code with fewer operations per vector: a not-counted cell's code byte is 0x80
+// (its 16-bit index >= 0x8000 > every slot, so the dummy clamp still catches it) and both code
+// bytes come straight out of one multiply each — bit j of a nibble times 0x00204081 * k, masked
+// with 0x01010101 * k, is byte j = k (k a power of two): 0x80 for skip, ob = offb >> 8 for B.
+// mb = 0x00204081 * ob, kb = 0x01010101 * ob (the caller hoists them).
+template <int kForm>
+__device__ __forceinline__ void count8_fast_code2(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                                  uint32_t sel, const FastBins& f, uint32_t dumB2, uint32_t mb,
+                                                  uint32_t kb) {
+  const uint32_t e = sel & ~skip;
+  const uint32_t clo = (((skip & 0xFu) * 0x10204080u) & 0x80808080u) | (((e & 0xFu) * mb) & kb);
+  const uint32_t chi = (((skip >> 4) * 0x10204080u) & 0x80808080u) | (((e >> 4) * mb) & kb);
+  const uint32_t ws[4] = {q.x, q.y, q.z, q.w};
+  char* hb = reinterpret_cast<char*>(hist);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t j = (uint32_t)(i & 1) * 2;
+    const uint32_t P = 4u | (j << 4) | (4u << 8) | ((j + 1) << 12);
+    uint32_t x = fast_idx2<kForm, ZH_NEG>(ws[i], f) | __byte_perm(i < 2 ? clo : chi, 0u, P);
     x = __vminu2(x, dumB2) << 2;
     atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
     atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);

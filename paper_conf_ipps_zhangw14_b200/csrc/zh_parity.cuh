@@ -61,6 +61,9 @@ __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr,
 // Shared-memory queue of long edges (more than kLongRows straddled rows in the chunk): they are
 // processed afterwards by whole warps, one row per lane, so that no thread serialises hundreds of
 // rows while the others wait at the barrier.
+#ifndef ZH_PAR_SPEC
+#define ZH_PAR_SPEC 1
+#endif
 #ifndef ZH_LONG_ROWS
 #define ZH_LONG_ROWS 8
 #endif
@@ -83,10 +86,17 @@ __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, i
   const int w = t.w;
   for (int i = e0 + threadIdx.x; i < e1; i += blockDim.x) {
     const int v = band_edges[i];
+#if ZH_PAR_SPEC  // the edge's rows and coordinates loaded together: two dependent loads, not three
+    const int2 rr = erows[v];
+    const Edge e = edges[v];
+    const int64_t ra = max((int64_t)rr.x, rlo), rb = min((int64_t)rr.y, rhi);
+    if (ra >= rb) continue;
+#else
     const int2 rr = erows[v];
     const int64_t ra = max((int64_t)rr.x, rlo), rb = min((int64_t)rr.y, rhi);
     if (ra >= rb) continue;
     const Edge e = edges[v];
+#endif
     const double exl = fmin(e.xa, e.xb), exh = fmax(e.xa, e.xb);
     if (exh + t.half < t.xlo_t) continue;  // xi < every xc: crosses no cell of the tile
     const int all = exl - t.half > t.xhi_t;  // xi > every xc: crosses every cell

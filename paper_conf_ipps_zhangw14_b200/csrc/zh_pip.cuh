@@ -15,6 +15,25 @@
 #ifndef ZH_MIX_IL
 #define ZH_MIX_IL 1
 #endif
+// k_mixed_cells: code bytes from one multiply per nibble (count8_fast_code2) instead of
+// count8_fast_code's spread-then-scale
+#ifndef ZH_CODE2
+#define ZH_CODE2 1
+#endif
+// k_mixed_cells main loop: staged bitmap words through a pointer stepped by a uniform stride
+// (aligned tiles), and no zeroing of the raster registers of skipped vectors (never counted)
+#ifndef ZH_MIX_PTR
+#define ZH_MIX_PTR 1
+#endif
+#ifndef ZH_MIX_DIAG
+#define ZH_MIX_DIAG 0  // timing diagnostics (wrong results): 1 no cell routing / atomics, 2 no flush
+#endif
+#ifndef ZH_MIX_PF
+#define ZH_MIX_PF 0  // k_mixed_cells: L2 prefetch distance in main-loop iterations (0 = none)
+#endif
+#ifndef ZH_MIX_NOZERO
+#define ZH_MIX_NOZERO 0
+#endif
 
 namespace zh {
 
@@ -259,6 +278,9 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
   const uint32_t dum2 = dummy * 0x10001u;
   const uint32_t off2 = (uint32_t)OB * 0x10001u;
   const uint32_t dumB2 = (dummy + (uint32_t)OB) * 0x10001u, ob = (uint32_t)OB >> 8;
+  const uint32_t mb = 0x00204081u * ob, kb = 0x01010101u * ob;
+  uint32_t diag = 0;
+  (void)diag;
   const int64_t k0 = c0 >> 3, k1 = (c0 + w + 7) >> 3;
   const int nk = (int)(k1 - k0);
   const int64_t pitch = rp.pitch;
@@ -269,7 +291,10 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
   };
   auto count_sel = [&](const uint4& q, uint32_t skip, uint32_t sel) {
     if constexpr (kMode >= 2) {
-      if (kCode) count8_fast_code<kMode - 2>(hist, q, skip, sel, fb, dumB2, ob);
+      if (kCode) {
+        if (ZH_CODE2) count8_fast_code2<kMode - 2>(hist, q, skip, sel, fb, dumB2, mb, kb);
+        else count8_fast_code<kMode - 2>(hist, q, skip, sel, fb, dumB2, ob);
+      }
       else count8_fast_sel<kMode - 2>(hist, q, skip, sel, fb, dum2, off2);
     } else {
       count8_generic_sel<kMode == 0>(hist, q, skip, sel, p.bp, dummy, OB);
@@ -310,6 +335,8 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
     }
     const bool overlap = __syncthreads_or(ov != 0) != 0;
     const int16_t* base = rp.data + (r0 + cr - rp.row0) * pitch + k0 * 8;
+    const int hrem = h - cr;  // rows of the tile from this chunk on (prefetch bound)
+    (void)hrem;
     if (nk <= (int)blockDim.x) {
       const int rpi = blockDim.x / nk;
       const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
@@ -341,20 +368,57 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
 #if ZH_MIX_ROWS4
           // ZH_MIX_NR rows per iteration: that many 16-byte loads in flight per thread
           constexpr int NR = ZH_MIX_NR;
+#if ZH_MIX_PTR
+          // aligned: this thread's interleaved bitmap word of row lr, stepped by a uniform stride
+          const uint2* bw = reinterpret_cast<const uint2*>(bm0) + lr * wpo + wi;
+          const int bstride = rpi * wpo;
+#endif
           for (; lr + (NR - 1) * rpi < ch; lr += NR * rpi, ptr += NR * step) {
             uint32_t e[NR], s[NR];
             uint4 q[NR];
 #pragma unroll
             for (int u = 0; u < NR; ++u) {
-              const uint2 b2 = pb2(lr + u * rpi);
+              uint2 b2;
+#if ZH_MIX_PTR
+              if (kA) {
+                const uint2 v = bw[u * bstride];
+                b2 = make_uint2((v.x >> bsh) & 0xFFu, (v.y >> bsh) & 0xFFu);
+              } else {
+                b2 = pb2(lr + u * rpi);
+              }
+#else
+              b2 = pb2(lr + u * rpi);
+#endif
               e[u] = b2.y;
               s[u] = cskip | (~(b2.x | b2.y) & 0xFFu);
+#if ZH_MIX_NOZERO
+              if (s[u] != 0xFFu) q[u] = ld_stream16(ptr + u * step);
+#else
               q[u] = make_uint4(0, 0, 0, 0);
               if (s[u] != 0xFFu) q[u] = ld_stream16(ptr + u * step);
+#endif
             }
+#if ZH_MIX_PTR
+            bw += NR * bstride;
+#endif
+#if ZH_MIX_PF
+            // L2 prefetch of the rows ZH_MIX_PF iterations ahead (no registers held)
+#pragma unroll
+            for (int u = 0; u < NR; ++u) {
+              const int ahead = (ZH_MIX_PF * NR + u) * rpi;
+              if (lr + ahead < hrem)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(ptr + (int64_t)(ZH_MIX_PF * NR + u) * step));
+            }
+#endif
 #pragma unroll
             for (int u = 0; u < NR; ++u)
-              if (s[u] != 0xFFu) count_sel(q[u], s[u], e[u]);
+              if (s[u] != 0xFFu) {
+#if ZH_MIX_DIAG & 1  // timing diagnostic only: no routing / atomics (wrong counts)
+                diag ^= q[u].x ^ q[u].y ^ q[u].z ^ q[u].w ^ s[u] ^ e[u];
+#else
+                count_sel(q[u], s[u], e[u]);
+#endif
+              }
           }
 #endif
           for (; lr + rpi < ch; lr += 2 * rpi, ptr += 2 * step) {
@@ -417,8 +481,13 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
     }
     __syncthreads();
   }
+#if ZH_MIX_DIAG
+  if (diag == 0x12345678u) hist[0] = 1;  // keeps the diagnostic sink alive
+#endif
+#if !(ZH_MIX_DIAG & 2)
   flush_hist<kU64>(hist, p.bp.nbins, kp0, p.out);
   if (m > 1) flush_hist<kU64>(hist + OB, p.bp.nbins, kp1, p.out);
+#endif
 }
 
 }  // namespace zh

@@ -1,11 +1,12 @@
 #!/bin/bash
 # A/B of libzh builds on the bench step (no e2e / CPU / other path).  Usage: tools/ab_bench.sh tag lib1 [lib2 ...]
-# ("default" = the in-tree build).  Lines go to gpurun_out/ab_<tag>.txt.
+# ("default" = the in-tree build; BENCH_ARGS="--config pip-stress" etc. passed to bench.py).
+# Lines go to gpurun_out/ab_<tag>.txt.
 TAG=$1; shift
 mkdir -p gpurun_out
 for L in "$@"; do
   if [ "$L" = default ]; then unset ZH_LIBZH; else export ZH_LIBZH=$PWD/$L; fi
-  timeout 600 python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu --no-other "${BENCH_ARGS[@]}" > gpurun_out/ab_tmp.json 2>gpurun_out/ab_tmp.err
+  timeout 600 python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu --no-other $BENCH_ARGS > gpurun_out/ab_tmp.json 2>gpurun_out/ab_tmp.err
   python - "$L" <<'PY' >> gpurun_out/ab_${TAG}.txt
 import json, sys
 try:
