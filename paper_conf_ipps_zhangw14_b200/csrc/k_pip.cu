@@ -65,11 +65,14 @@ __global__ void __launch_bounds__(kPipThreads, ZH_PIP_MINB) k_pip_cells(PipP p) 
 #ifndef ZH_MIX_CODE
 #define ZH_MIX_CODE 1  // k_mixed_cells: code-byte routing with B at a power-of-two offset (packed bins)
 #endif
+#ifndef ZH_MIX_FLAT
+#define ZH_MIX_FLAT 1  // k_mixed_cells: flat layout (whole-tile bitmaps, added code bytes) when it fits
+#endif
 #ifndef ZH_MIX_MINB
 #define ZH_MIX_MINB 4
 #endif
 // Tile groups of <= 2 pairs (fused path): each cell read once per group (zh_pip.cuh).
-template <int kMode, bool kU64, bool kCode>
+template <int kMode, bool kU64, int kCode>
 __global__ void __launch_bounds__(ZH_MIX_THREADS, ZH_MIX_MINB) k_mixed_cells(PipP p) {
   if (p.n_dev && (int64_t)blockIdx.x >= *p.n_dev) return;
   extern __shared__ __align__(16) uint32_t sh[];
@@ -161,20 +164,40 @@ static int mixed_rows(const Ctx& c) {
 }
 
 // Shared-memory layout of k_mixed_cells: histogram A at word 0, B at word *offb, the two staged
-// bitmaps at word *bmo.  With packed bins, B sits at a power of two (code bytes route the cells,
-// count8_fast_code) and the bitmaps fill the gap below it when they fit; otherwise B follows A.
+// bitmaps (*rows rows of each pair) at word *bmo; *code = the routing form (mixed_cells_body's kCode).
+//  2 (flat, preferred): B right after A at a multiple of 256 words, the whole tile's bitmaps
+//    after B (one staging round per group instead of one per 128 rows), code bytes added; only
+//    while the CTA stays within 56 KB (4 CTAs per SM) and the 16-bit indices cannot wrap;
+//  1: B at a power of two (OR-ed code bytes), 128-row bitmap chunks in the gap below it;
+//  0: B right after A, offsets added per cell.
 // Returns the bytes, or 0 when the grouped form does not apply (two histograms must fit the CTA,
 // and the packed forms need 16-bit byte offsets over both).
-static size_t mixed_layout(const Ctx& c, int* offb, int* bmo, bool* code) {
+static size_t mixed_layout(const Ctx& c, int* offb, int* bmo, int* code, int* rows) {
   const int hw = hist_words(c.bp.nbins);
-  const int bmw = 2 * mixed_rows(c) * ((c.rp.T + 31) / 32);
+  const int wpo = (c.rp.T + 31) / 32;
   const bool packed = pip_mode(c) >= 2;
-  int ob = 256;
-  while (ob < hw) ob *= 2;
   const FastBins fb = make_fast_bins(c.bp);
   const int nod_idx = 0xFFFF - (int)(fb.Cb2 & 0xFFFFu);
-  *code = ZH_MIX_CODE && packed && (ob + hw) * 4 < 65536 && (!fb.bias || nod_idx >= ob + hw);
-  if (*code) {
+  {
+    const int ob = (hw + 255) & ~255;
+    const int bo = (ob + hw + 3) & ~3;
+    const size_t words = (size_t)bo + 2 * (size_t)c.rp.T * wpo;
+    if (ZH_MIX_FLAT && packed && pip_mode(c) != 3 && (ob >> 8) < 0x40 && ob + hw < 0x4000 &&
+        (!fb.bias || (nod_idx >= ob + hw && nod_idx + 0x4000 <= 0xFFFF)) && words * 4 <= 56 * 1024) {
+      *code = 2;
+      *offb = ob;
+      *bmo = bo;
+      *rows = c.rp.T;
+      return words * 4;
+    }
+  }
+  *rows = mixed_rows(c);
+  const int bmw = 2 * *rows * wpo;
+  int ob = 256;
+  while (ob < hw) ob *= 2;
+  const bool c1 = ZH_MIX_CODE && packed && (ob + hw) * 4 < 65536 && (!fb.bias || nod_idx >= ob + hw);
+  *code = c1 ? 1 : 0;
+  if (c1) {
     *offb = ob;
     *bmo = (hw + bmw <= ob) ? hw : ob + hw;
   } else {
@@ -183,26 +206,24 @@ static size_t mixed_layout(const Ctx& c, int* offb, int* bmo, bool* code) {
   }
   const size_t words = std::max<size_t>((size_t)*offb + hw, (size_t)*bmo + bmw);
   if (words * 4 > 200 * 1024) return 0;
-  if (packed && !*code && 2 * (size_t)hw * 4 >= 65536) return 0;
+  if (packed && !c1 && 2 * (size_t)hw * 4 >= 65536) return 0;
   return words * 4;
 }
 
 size_t mixed_smem(Ctx& c) {
-  int ob, bo;
-  bool code;
-  return mixed_layout(c, &ob, &bo, &code);
+  int ob, bo, code, rows;
+  return mixed_layout(c, &ob, &bo, &code, &rows);
 }
 
 cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64_t grid, const int64_t* n_dev) {
   if (grid == 0) return cudaSuccess;
   PipP p = pip_params(c, pairs, n_dev);
   p.grp = grp;
-  p.rcc = mixed_rows(c);
-  bool code = false;
-  const size_t smem = mixed_layout(c, &p.offb, &p.bmo, &code);
+  int code = 0;
+  const size_t smem = mixed_layout(c, &p.offb, &p.bmo, &code, &p.rcc);
   void (*k)(PipP);
-#define ZH_MIX_K(M) (c.out_u64 ? (code ? k_mixed_cells<M, true, true> : k_mixed_cells<M, true, false>) \
-                               : (code ? k_mixed_cells<M, false, true> : k_mixed_cells<M, false, false>))
+#define ZH_MIX_K1(M, U) (code == 2 ? k_mixed_cells<M, U, 2> : code == 1 ? k_mixed_cells<M, U, 1> : k_mixed_cells<M, U, 0>)
+#define ZH_MIX_K(M) (c.out_u64 ? ZH_MIX_K1(M, true) : ZH_MIX_K1(M, false))
   switch (pip_mode(c)) {
     case 0: k = ZH_MIX_K(0); break;
     case 1: k = ZH_MIX_K(1); break;
@@ -211,6 +232,7 @@ cudaError_t launch_mixed_cells(Ctx& c, const int2* pairs, const int2* grp, int64
     default: k = ZH_MIX_K(4); break;
   }
 #undef ZH_MIX_K
+#undef ZH_MIX_K1
   prep_kernel(k, smem);
   k<<<(unsigned)grid, ZH_MIX_THREADS, smem, c.stream>>>(p);
   c.launches += 1;

@@ -301,6 +301,31 @@ __device__ __forceinline__ void count8_fast_code2(uint32_t* __restrict__ hist, c
   }
 }
 
+// Flat layout of k_mixed_cells (B right after A, at a multiple of 256 words, so that a group's
+// whole-tile bitmaps fit beside both histograms): the code byte is ADDED to the cell's 16-bit
+// index — 0 (A), kB = offb >> 8 (B), 0x40 (not counted: index >= 0x4000, above every slot, the
+// dummy clamp catches it).  kForm 0 or 2 only; the caller guarantees offb + hist_words < 0x4000
+// and that a biased nodata index plus 0x40 << 8 stays below 2^16 (no half wraps, so the add of
+// both halves is one 32-bit add).
+template <int kForm>
+__device__ __forceinline__ void count8_fast_code3(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,
+                                                  uint32_t sel, const FastBins& f, uint32_t dumB2, uint32_t kB) {
+  const uint32_t e = sel & ~skip;
+  const uint32_t clo = (((skip & 0xFu) * 0x08102040u) & 0x40404040u) | ((((e & 0xFu) * 0x00204081u) & 0x01010101u) * kB);
+  const uint32_t chi = (((skip >> 4) * 0x08102040u) & 0x40404040u) | ((((e >> 4) * 0x00204081u) & 0x01010101u) * kB);
+  const uint32_t ws[4] = {q.x, q.y, q.z, q.w};
+  char* hb = reinterpret_cast<char*>(hist);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t j = (uint32_t)(i & 1) * 2;
+    const uint32_t P = 4u | (j << 4) | (4u << 8) | ((j + 1) << 12);
+    uint32_t x = fast_idx2<kForm, ZH_NEG>(ws[i], f) + __byte_perm(i < 2 ? clo : chi, 0u, P);
+    x = __vminu2(x, dumB2) << 2;
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
+    atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);
+  }
+}
+
 // Generic path (any width / lo / nbins): same layout, scalar mapping, per-cell atomics.
 template <bool kW1>
 __device__ __forceinline__ void count8_generic(uint32_t* __restrict__ hist, const uint4& q, uint32_t skip,

@@ -248,9 +248,10 @@ __device__ __forceinline__ uint2 bits8_il(const uint2* __restrict__ row, int wpr
 // one atomic per cell, whatever m).  Otherwise (overlapping polygons, cover mode) every vector is
 // counted once per pair.  The branch is uniform over the CTA (__syncthreads_or of the overlap).
 // `sh` holds 2 hist_words(nbins) + 2 rcc * wpo words.
-// kCode: B at a power-of-two offset, cells routed by code bytes (count8_fast_code); otherwise
-// count8_fast_sel / count8_generic_sel add the offset.
-template <int kMode, bool kU64, bool kCode>
+// kCode: 1 — B at a power-of-two offset, cells routed by OR-ed code bytes (count8_fast_code2);
+// 2 — flat layout, B right after A and the whole tile's bitmaps staged at once, ADDED code bytes
+// (count8_fast_code3); 0 — count8_fast_sel / count8_generic_sel add the offset.
+template <int kMode, bool kU64, int kCode>
 __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint32_t* __restrict__ sh) {
   const int HW = hist_words(p.bp.nbins);
   const int2 gr = p.grp[g];
@@ -291,7 +292,9 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
   };
   auto count_sel = [&](const uint4& q, uint32_t skip, uint32_t sel) {
     if constexpr (kMode >= 2) {
-      if (kCode) {
+      if (kCode == 2) {
+        if constexpr (kMode - 2 != 1) count8_fast_code3<kMode - 2>(hist, q, skip, sel, fb, dumB2, ob);
+      } else if (kCode == 1) {
         if (ZH_CODE2) count8_fast_code2<kMode - 2>(hist, q, skip, sel, fb, dumB2, mb, kb);
         else count8_fast_code<kMode - 2>(hist, q, skip, sel, fb, dumB2, ob);
       }

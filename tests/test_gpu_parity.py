@@ -161,7 +161,10 @@ def test_flipped_geotransforms(tiny, cuda_device, flip):
                                                          # (tiny: -157..401): clamp counts them in
                                                          # bin 0, drop drops them
                                                          (0, 1, 256, False, -100), (0, 1, 256, True, -100),
-                                                         (-50, 1, 5000, False, -120), (-150, 1, 600, False, -151)])
+                                                         (-50, 1, 5000, False, -120), (-150, 1, 600, False, -151),
+                                                         # k_mixed_cells layouts: flat without nodata
+                                                         # (kForm 0), power-of-two B (7,000 bins)
+                                                         (0, 1, 4000, False, None), (0, 1, 7000, False, -32768)])
 def test_bin_mappings(tiny, cuda_device, lo, width, nbins, drop, nodata):
     cfg, P, R, _ = tiny
     H = oracle.o1(R, cfg.gt, P, oracle.make_bins(nbins, lo=lo, width=width, nodata=nodata, oor_drop=drop))
