@@ -390,6 +390,18 @@ cudaError_t launch_check_counts(Ctx& c, const int64_t* counts, const int64_t* wa
   return cudaGetLastError();
 }
 
+// Threads per CTA of the one-CTA-per-polygon step-2 kernels (k_mbb_edges, k_poly_bands, k_mark):
+// about one edge per thread or more — 256 for county-sized rings (CONUS: ~3,000 vertices), fewer
+// for small ones (PIP-stress: ~760), where a 256-thread CTA mostly waits at its barriers.
+static int s2_threads(const Ctx& c) {
+#ifdef ZH_S2_THREADS
+  return ZH_S2_THREADS;
+#else
+  const int64_t avg = c.P > 0 ? (int64_t)c.V / c.P : 0;
+  return avg >= 1536 ? 256 : (avg >= 384 ? 128 : 64);
+#endif
+}
+
 cudaError_t launch_pairs_phase1(Ctx& c) {
   cudaError_t e;
   const int V = c.V, P = c.P;
@@ -413,7 +425,7 @@ cudaError_t launch_pairs_phase1(Ctx& c) {
     prep_kernel(k_classify, 0);
   }
   if (P > 0) {
-    k_mbb_edges<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
+    k_mbb_edges<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_x.as<double>(),
                                          c.d_y.as<double>(), c.geo, c.rp, c.d_mbb.as<int4>(), c.d_ncand.as<int64_t>(),
                                          c.d_nband.as<int64_t>(), rA, rB, c.d_edges.as<Edge>(), c.d_erows.as<int2>(),
                                          c.d_counts.as<int64_t>() + 2);
@@ -442,7 +454,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   // The band (polygon, tile-row) edge lists.
   cudaMemsetAsync(c.d_band_cnt.p, 0, sizeof(int32_t) * ((size_t)nb + 1), c.stream);
   if (V > 0 && nb > 0) {
-    k_poly_bands<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
+    k_poly_bands<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
                                           c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 0,
                                           c.d_band_cnt.as<int32_t>(), nullptr, nullptr, c.d_band_poly.as<int32_t>());
     c.launches += 1;
@@ -452,7 +464,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
       return e;
     cudaMemcpyAsync(c.d_band_cur.p, c.d_band_off.p, sizeof(int32_t) * (size_t)nb, cudaMemcpyDeviceToDevice, c.stream);
     if (V > 0) {
-      k_poly_bands<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
+      k_poly_bands<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
                                             c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 1,
                                             c.d_band_cur.as<int32_t>(), c.d_band_off.as<int32_t>(),
                                             c.d_band_edges.as<int32_t>(), nullptr);
@@ -466,7 +478,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
     } else {
       cudaMemsetAsync(c.d_class.p, 0, (size_t)nc, c.stream);
       if (V > 0) {
-        k_mark<<<P, 256, 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_edges.as<Edge>(), c.geo,
+        k_mark<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_edges.as<Edge>(), c.geo,
                                        c.rp, c.d_mbb.as<int4>(),
                                                       c.d_cand_off.as<int64_t>(), c.d_class.as<uint8_t>());
         c.launches += 1;
