@@ -319,8 +319,8 @@ __device__ __forceinline__ void count8_fast_code3(uint32_t* __restrict__ hist, c
   for (int i = 0; i < 4; ++i) {
     const uint32_t j = (uint32_t)(i & 1) * 2;
     const uint32_t P = 4u | (j << 4) | (4u << 8) | ((j + 1) << 12);
-    uint32_t x = fast_idx2<kForm, ZH_NEG>(ws[i], f) + __byte_perm(i < 2 ? clo : chi, 0u, P);
-    x = __vminu2(x, dumB2) << 2;
+    // per-half add of the code, then the dummy clamp: one VIADDMNMX
+    uint32_t x = __vminu2(__vadd2(fast_idx2<kForm, ZH_NEG>(ws[i], f), __byte_perm(i < 2 ? clo : chi, 0u, P)), dumB2) << 2;
     atomicAdd(reinterpret_cast<uint32_t*>(hb + (x & 0xFFFFu)), 1u);
     atomicAdd(reinterpret_cast<uint32_t*>(hb + (x >> 16)), 1u);
   }
