@@ -167,27 +167,35 @@ __global__ void __launch_bounds__(256) k_mbb_edges(const int32_t* __restrict__ p
 
 // Band lists, one CTA per polygon: its vertices (= edges) are contiguous, and the counters of its
 // bands (one per tile row of its MBB) live in shared memory, so the heavily repeated increments of
-// consecutive edges never leave the SM.  mode 0: counts -> band_cnt; mode 1: fill band_edges from
-// band_off.  Polygons with more bands than kSmemBands use global atomics directly.
-constexpr int kSmemBands = 4096;
+// consecutive edges never leave the SM.  mode 0: counts -> band_cnt, and band_first = how many of
+// them straddle the band's FIRST row (the row k_classify tests; -1: not sorted, polygons with more
+// bands than kSmemBands, which use global atomics directly); mode 1: fill band_edges from band_off,
+// those first-row edges at the front of the list.
+constexpr int kSmemBands = 2048;
 __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
                                                     const int2* __restrict__ erows, const int4* __restrict__ mbb,
                                                     const int64_t* __restrict__ band_base, int T, int mode,
                                                     int32_t* __restrict__ band_cnt, const int32_t* __restrict__ band_off,
-                                                    int32_t* __restrict__ band_edges, int32_t* __restrict__ band_poly) {
+                                                    int32_t* __restrict__ band_edges, int32_t* __restrict__ band_poly,
+                                                    int32_t* __restrict__ band_first) {
   __shared__ int32_t sc[kSmemBands];
+  __shared__ int32_t sb[kSmemBands];  // first-row edges (mode 0) / cursor of the rest (mode 1)
   const int k = blockIdx.x;
   const int4 m = mbb[k];
   if (m.x > m.y) return;
   const int nb = m.w - m.z + 1;
   const int64_t bb = band_base[k];
   const bool in_smem = nb <= kSmemBands;
-  int32_t* cnt = in_smem ? sc : nullptr;
   if (mode == 0)
     for (int i = threadIdx.x; i < nb; i += blockDim.x) band_poly[bb + i] = k;  // band -> polygon
   if (in_smem) {
-    for (int i = threadIdx.x; i < nb; i += blockDim.x) sc[i] = mode == 0 ? 0 : band_off[bb + i];
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) {
+      sc[i] = 0;
+      sb[i] = 0;
+    }
     __syncthreads();
+  } else if (mode == 0) {
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) band_first[bb + i] = -1;
   }
   const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
   for (int v = vb + threadIdx.x; v < ve; v += blockDim.x) {
@@ -195,18 +203,30 @@ __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ 
     if (rr.x >= rr.y) continue;
     for (int tr = rr.x / T; tr <= (rr.y - 1) / T; ++tr) {
       const int i = tr - m.z;
+      const int64_t r = (int64_t)tr * T;  // the band's first row
+      const bool first = rr.x <= r && r < rr.y;
       if (mode == 0) {
-        if (in_smem) atomicAdd(&cnt[i], 1);
-        else atomicAdd(&band_cnt[bb + i], 1);
-      } else {
-        const int pos = in_smem ? atomicAdd(&cnt[i], 1) : atomicAdd(&band_cnt[bb + i], 1);  // band_cnt = cursors
+        if (in_smem) {
+          atomicAdd(&sc[i], 1);
+          if (first) atomicAdd(&sb[i], 1);
+        } else {
+          atomicAdd(&band_cnt[bb + i], 1);
+        }
+      } else if (in_smem) {
+        const int pos = first ? band_off[bb + i] + atomicAdd(&sc[i], 1)
+                              : band_off[bb + i] + band_first[bb + i] + atomicAdd(&sb[i], 1);
         band_edges[pos] = v;
+      } else {
+        band_edges[atomicAdd(&band_cnt[bb + i], 1)] = v;  // band_cnt = cursors
       }
     }
   }
-  if (mode == 0 && in_smem) {
+  if (in_smem && mode == 0) {
     __syncthreads();
-    for (int i = threadIdx.x; i < nb; i += blockDim.x) band_cnt[bb + i] = sc[i];
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) {
+      band_cnt[bb + i] = sc[i];
+      band_first[bb + i] = sb[i];
+    }
   }
 }
 
@@ -261,7 +281,8 @@ constexpr int kClassifyWarps = 4;
 __global__ void __launch_bounds__(32 * kClassifyWarps) k_classify(
     const Edge* __restrict__ edges, const int2* __restrict__ erows, const int32_t* __restrict__ band_off,
     const int32_t* __restrict__ band_edges, const int64_t* __restrict__ band_base,
-    const int32_t* __restrict__ band_poly, int64_t n_bands, Geo g, RasterP rp, const int4* __restrict__ mbb,
+    const int32_t* __restrict__ band_poly, const int32_t* __restrict__ band_first, int64_t n_bands, Geo g, RasterP rp,
+    const int4* __restrict__ mbb,
     const int64_t* __restrict__ cand_off, uint8_t* __restrict__ cls, int dwords) {
   extern __shared__ uint32_t Dall[];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -278,7 +299,8 @@ __global__ void __launch_bounds__(32 * kClassifyWarps) k_classify(
   const int nd = (wk >> 5) + 1;
   for (int i = lane; i < nd; i += 32) D[i] = 0;
   __syncwarp();
-  const int e0 = band_off[band], e1 = band_off[band + 1];
+  const int e0 = band_off[band], nf = band_first[band];
+  const int e1 = nf >= 0 ? e0 + nf : band_off[band + 1];  // the edges straddling row rrep come first
   for (int i = e0 + lane; i < e1; i += 32) {
     const int v = band_edges[i];
     const int2 rr = erows[v];
@@ -448,6 +470,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   if ((e = c.d_band_cur.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
   if ((e = c.d_band_edges.ensure(sizeof(int32_t) * (size_t)ne)) != cudaSuccess) return e;
   if ((e = c.d_band_poly.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
+  if ((e = c.d_band_first.ensure(sizeof(int32_t) * ((size_t)nb + 1))) != cudaSuccess) return e;
   if ((e = c.d_class.ensure((size_t)nc)) != cudaSuccess) return e;
   if ((e = c.d_flags.ensure(sizeof(uint64_t) * (size_t)nc)) != cudaSuccess) return e;
   if ((e = c.d_flag_pos.ensure(sizeof(uint64_t) * (size_t)nc)) != cudaSuccess) return e;
@@ -456,7 +479,8 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   if (V > 0 && nb > 0) {
     k_poly_bands<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
                                           c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 0,
-                                          c.d_band_cnt.as<int32_t>(), nullptr, nullptr, c.d_band_poly.as<int32_t>());
+                                          c.d_band_cnt.as<int32_t>(), nullptr, nullptr, c.d_band_poly.as<int32_t>(),
+                                          c.d_band_first.as<int32_t>());
     c.launches += 1;
   }
   if (nb > 0) {
@@ -467,7 +491,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
       k_poly_bands<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
                                             c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 1,
                                             c.d_band_cur.as<int32_t>(), c.d_band_off.as<int32_t>(),
-                                            c.d_band_edges.as<int32_t>(), nullptr);
+                                            c.d_band_edges.as<int32_t>(), nullptr, c.d_band_first.as<int32_t>());
       c.launches += 1;
     }
   }
@@ -490,7 +514,8 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
       prep_kernel(k_classify, smem);
       k_classify<<<(unsigned)((nb + nw - 1) / nw), 32 * nw, smem, c.stream>>>(
           c.d_edges.as<Edge>(), c.d_erows.as<int2>(), c.d_band_off.as<int32_t>(), c.d_band_edges.as<int32_t>(),
-          c.d_band_base.as<int64_t>(), c.d_band_poly.as<int32_t>(), nb, c.geo, c.rp, c.d_mbb.as<int4>(),
+          c.d_band_base.as<int64_t>(), c.d_band_poly.as<int32_t>(), c.d_band_first.as<int32_t>(), nb, c.geo, c.rp,
+          c.d_mbb.as<int4>(),
           c.d_cand_off.as<int64_t>(), c.d_class.as<uint8_t>(), dwords);
       c.launches += 1;
     }

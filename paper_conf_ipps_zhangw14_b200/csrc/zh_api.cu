@@ -427,7 +427,7 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
                       &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats,
-                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_band_poly, &c->d_flag, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
+                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_band_poly, &c->d_band_first, &c->d_flag, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
   for (auto* b : bufs) b->release();
   ZH_TR("release");
   for (int i = 0; i < 16; ++i)
@@ -456,7 +456,7 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
                             &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats,
-                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_band_poly, &c.d_flag, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
+                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_band_poly, &c.d_band_first, &c.d_flag, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;
