@@ -64,48 +64,13 @@ __device__ __forceinline__ int2 straddle_rows(const Geo& g, double ya, double yb
   return make_int2((int)ra, (int)rb);
 }
 
-// One CTA per polygon: for every vertex v of its rings, the edge v -> next(v) (implicit closure) in
-// canonical orientation and its exact straddled row interval within the shard; the number of
-// (edge, tile row) band entries is added to *n_entries.  Polygons whose tile rectangle misses the
-// shard (empty MBB) are skipped: nothing downstream reads their edges.  (Rings are contiguous, so
-// no search is needed.)
-__device__ __forceinline__ void edges_body(int k, const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
-                                           const double* __restrict__ x, const double* __restrict__ y, const Geo& g,
-                                           int64_t rA, int64_t rB, int T, Edge* __restrict__ edges,
-                                           int2* __restrict__ erows, int64_t* __restrict__ n_entries) {
-  int span = 0;
-  for (int ring = pro[k]; ring < pro[k + 1]; ++ring) {
-    const int a = rvo[ring], b = rvo[ring + 1];
-    for (int v = a + threadIdx.x; v < b; v += blockDim.x) {
-      const int nxt = (v + 1 < b) ? v + 1 : a;
-      const double x0 = x[v], y0 = y[v], x1 = x[nxt], y1 = y[nxt];
-      Edge e;
-      if (y0 <= y1) { e.xa = x0; e.ya = y0; e.xb = x1; e.yb = y1; }
-      else          { e.xa = x1; e.ya = y1; e.xb = x0; e.yb = y0; }
-      edges[v] = e;
-      const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
-      erows[v] = rr;
-      span += (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
-    }
-  }
-  for (int o = 16; o > 0; o >>= 1) span += __shfl_xor_sync(0xffffffffu, span, o);
-  if ((threadIdx.x & 31) == 0 && span) atomicAdd(reinterpret_cast<unsigned long long*>(n_entries),
-                                                 (unsigned long long)span);
-}
-
 // MBB of polygon k's vertices -> covered tile rectangle (global tile indices), clipped to the raster
-// columns and the shard rows.  Empty -> (1, 0, 1, 0).  Returned to every thread of the CTA.
-__device__ __forceinline__ int4 mbb_body(int k, const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
-                                         const double* __restrict__ x, const double* __restrict__ y, const Geo& g,
-                                         const RasterP& rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
-                                         int64_t* __restrict__ nband) {
+// columns and the shard rows, from each thread's partial min / max.  Empty -> (1, 0, 1, 0).
+// Returned to every thread of the CTA.
+__device__ __forceinline__ int4 mbb_reduce(int k, int nv, double xmn, double xmx, double ymn, double ymx, const Geo& g,
+                                           const RasterP& rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
+                                           int64_t* __restrict__ nband) {
   __shared__ int4 s_m;
-  const int vb = rvo[pro[k]], ve = rvo[pro[k + 1]];
-  double xmn = INFINITY, xmx = -INFINITY, ymn = INFINITY, ymx = -INFINITY;
-  for (int i = vb + threadIdx.x; i < ve; i += blockDim.x) {
-    xmn = fmin(xmn, x[i]); xmx = fmax(xmx, x[i]);
-    ymn = fmin(ymn, y[i]); ymx = fmax(ymx, y[i]);
-  }
   __shared__ double s[4][8];
   for (int o = 16; o > 0; o >>= 1) {
     xmn = fmin(xmn, __shfl_xor_sync(0xffffffffu, xmn, o));
@@ -123,7 +88,7 @@ __device__ __forceinline__ int4 mbb_body(int k, const int32_t* __restrict__ pro,
     }
     int4 m = make_int4(1, 0, 1, 0);
     int64_t nc = 0, nb = 0;
-    if (ve > vb) {
+    if (nv > 0) {
       double ca = (xmn - g.gt0) / g.gt1, cb = (xmx - g.gt0) / g.gt1;
       double ra = (ymn - g.gt3) / g.gt5, rb = (ymx - g.gt3) / g.gt5;
       if (ca > cb) { double t = ca; ca = cb; cb = t; }
@@ -150,9 +115,12 @@ __device__ __forceinline__ int4 mbb_body(int k, const int32_t* __restrict__ pro,
   return s_m;
 }
 
-// One CTA per polygon (step 2, first pass): the MBB's tile rectangle, then — when it meets the
-// shard — the canonical edges and their exact straddled rows (the vertices are read twice, the
-// second time from L1/L2).
+// One CTA per polygon (step 2, first pass), one pass over its vertices: each vertex v starts the
+// edge v -> next(v) (implicit closure), written in canonical orientation with its exact straddled
+// row interval within the shard, and joins the MBB's partial min / max; then the MBB's tile
+// rectangle.  The polygon's (edge, tile row) band entries count towards *n_entries only when the
+// rectangle meets the shard (nothing downstream reads the edges of the others).  (Rings are
+// contiguous, so no search is needed.)
 __global__ void __launch_bounds__(256) k_mbb_edges(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
                                                    const double* __restrict__ x, const double* __restrict__ y, Geo g,
                                                    RasterP rp, int4* __restrict__ mbb, int64_t* __restrict__ ncand,
@@ -160,9 +128,30 @@ __global__ void __launch_bounds__(256) k_mbb_edges(const int32_t* __restrict__ p
                                                    Edge* __restrict__ edges, int2* __restrict__ erows,
                                                    int64_t* __restrict__ n_entries) {
   const int k = blockIdx.x;
-  const int4 m = mbb_body(k, pro, rvo, x, y, g, rp, mbb, ncand, nband);
+  const int T = rp.T;
+  double xmn = INFINITY, xmx = -INFINITY, ymn = INFINITY, ymx = -INFINITY;
+  int span = 0;
+  for (int ring = pro[k]; ring < pro[k + 1]; ++ring) {
+    const int a = rvo[ring], b = rvo[ring + 1];
+    for (int v = a + threadIdx.x; v < b; v += blockDim.x) {
+      const int nxt = (v + 1 < b) ? v + 1 : a;
+      const double x0 = x[v], y0 = y[v], x1 = x[nxt], y1 = y[nxt];
+      xmn = fmin(xmn, x0); xmx = fmax(xmx, x0);
+      ymn = fmin(ymn, y0); ymx = fmax(ymx, y0);
+      Edge e;
+      if (y0 <= y1) { e.xa = x0; e.ya = y0; e.xb = x1; e.yb = y1; }
+      else          { e.xa = x1; e.ya = y1; e.xb = x0; e.yb = y0; }
+      edges[v] = e;
+      const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
+      erows[v] = rr;
+      span += (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
+    }
+  }
+  const int4 m = mbb_reduce(k, rvo[pro[k + 1]] - rvo[pro[k]], xmn, xmx, ymn, ymx, g, rp, mbb, ncand, nband);
   if (m.x > m.y) return;
-  edges_body(k, pro, rvo, x, y, g, rA, rB, rp.T, edges, erows, n_entries);
+  for (int o = 16; o > 0; o >>= 1) span += __shfl_xor_sync(0xffffffffu, span, o);
+  if ((threadIdx.x & 31) == 0 && span) atomicAdd(reinterpret_cast<unsigned long long*>(n_entries),
+                                                 (unsigned long long)span);
 }
 
 // Band lists, one CTA per polygon: its vertices (= edges) are contiguous, and the counters of its
