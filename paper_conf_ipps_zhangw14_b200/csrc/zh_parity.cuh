@@ -61,6 +61,9 @@ __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr,
 // Shared-memory queue of long edges (more than kLongRows straddled rows in the chunk): they are
 // processed afterwards by whole warps, one row per lane, so that no thread serialises hundreds of
 // rows while the others wait at the barrier.
+#ifndef ZH_PAR_DYN
+#define ZH_PAR_DYN 1  // k_parity: band edges claimed dynamically (atomic counter) after the first
+#endif
 #ifndef ZH_PAR_SPEC
 #define ZH_PAR_SPEC 1
 #endif
@@ -71,6 +74,7 @@ constexpr int kLongRows = ZH_LONG_ROWS;
 constexpr int kLongQ = 128;
 struct LongQ {
   int n;
+  int next;  // ZH_PAR_DYN: band edges claimed beyond the first blockDim.x
   int4 e[kLongQ];  // (edge, ra, rb, kind: 0 compute, 1 crosses every cell)
 };
 
@@ -84,7 +88,13 @@ __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, i
                                                     const Geo& g, const TileGeom& t, int64_t rlo, int64_t rhi,
                                                     LongQ* q) {
   const int w = t.w;
+#if ZH_PAR_DYN
+  // the first edge of each thread by index, the rest claimed one at a time (threads whose edges
+  // straddle few rows or miss the tile take more of them: no tail at the barrier below)
+  for (int i = e0 + threadIdx.x; i < e1; i = e0 + (int)blockDim.x + atomicAdd(&q->next, 1)) {
+#else
   for (int i = e0 + threadIdx.x; i < e1; i += blockDim.x) {
+#endif
     const int v = band_edges[i];
 #if ZH_PAR_SPEC  // the edge's rows and coordinates loaded together: two dependent loads, not three
     const int2 rr = erows[v];
@@ -116,7 +126,10 @@ __device__ __forceinline__ void crossings_to_bitmap(uint32_t* __restrict__ bm, i
   __syncthreads();
   const int nq = min(q->n, kLongQ);
   __syncthreads();                 // every thread has read the count ...
-  if (threadIdx.x == 0) q->n = 0;  // ... so it can be reset for the next call
+  if (threadIdx.x == 0) {  // ... so it can be reset for the next call
+    q->n = 0;
+    q->next = 0;
+  }
   const int lane = threadIdx.x & 31, nw = blockDim.x >> 5;
   for (int qi = threadIdx.x >> 5; qi < nq; qi += nw) {
     const int4 it = q->e[qi];

@@ -77,7 +77,10 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev);  // k_pip.cu
 template <bool kRep>
 __device__ __forceinline__ void parity_pair_body(const PipP& p, int64_t pair_idx, uint32_t* __restrict__ bm,
                                                  LongQ* lq) {
-  if (threadIdx.x == 0) lq->n = 0;
+  if (threadIdx.x == 0) {
+    lq->n = 0;
+    lq->next = 0;
+  }
   const RasterP& rp = p.rp;
   const Geo& g = p.g;
   const int2 pr = p.isect[pair_idx];
