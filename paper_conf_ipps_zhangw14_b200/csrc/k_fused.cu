@@ -70,7 +70,7 @@ __global__ void k_pure_fill(const int2* __restrict__ inside, int64_t n, const ui
 }
 
 __device__ __forceinline__ int64_t tile_cells(const RasterP& rp, int tile) {
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int trl = tile_row(rp, tile), tc = tile - trl * rp.TC;
   const int64_t r0 = (int64_t)(rp.tr0 + trl) * rp.T, c0 = (int64_t)tc * rp.T;
   return min((int64_t)rp.T, rp.row0 + rp.nrows - r0) * min((int64_t)rp.T, rp.cols - c0);
 }
@@ -241,7 +241,7 @@ __global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
   __syncthreads();
   for (int j = 0; j < nrun; ++j) {
     const int tile = s_tile[j];
-    const int trl = tile / f.rp.TC, tc = tile - trl * f.rp.TC;
+    const int trl = tile_row(f.rp, tile), tc = tile - trl * f.rp.TC;
     tile_histogram<kMode>(sh, f.rp, f.bp, f.fb, trl, tc);
     if (s_flush[j]) {  // uniform over the CTA
       __syncthreads();

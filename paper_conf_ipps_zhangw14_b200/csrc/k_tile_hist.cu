@@ -22,7 +22,7 @@ __global__ void __launch_bounds__(512, 3) k_tile_hist(RasterP rp, BinP bp, FastB
   extern __shared__ __align__(16) uint32_t sh[];
   const int HW = hist_words(bp.nbins);
   const int tile = blockIdx.x;
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int trl = tile_row(rp, tile), tc = tile - trl * rp.TC;
   for (int i = threadIdx.x * 4; i < HW; i += blockDim.x * 4)
     *reinterpret_cast<uint4*>(&sh[i]) = make_uint4(0, 0, 0, 0);
   __syncthreads();

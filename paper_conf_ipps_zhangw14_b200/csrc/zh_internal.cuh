@@ -364,6 +364,24 @@ struct RasterP {
   const int16_t* data;  // points at row `row0` of the full raster (device)
   int64_t rows, cols, pitch, row0, nrows;
   int32_t T, TC, tr0, TRn;  // tile size, tile columns, first tile row, tile rows in shard
+  uint32_t tc_mul, tc_sh;   // tile / TC by multiply-high (set_tc_div; Granlund-Montgomery round-up)
 };
+
+// tc_mul / tc_sh for an exact n / TC, n < 2^31, with one multiply-high instead of a division loop.
+__host__ inline void set_tc_div(RasterP& rp) {
+  const uint32_t d = (uint32_t)rp.TC;
+  uint32_t l = 0;
+  while ((1ull << l) < d) ++l;  // ceil(log2 d)
+  rp.tc_sh = l;
+  rp.tc_mul = l == 0 ? 0u : (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+}
+
+// (tile row, tile column) of a shard-local tile index
+__device__ __forceinline__ int tile_row(const RasterP& rp, int tile) {
+  const uint32_t n = (uint32_t)tile;
+  if (rp.tc_sh == 0) return tile;
+  const uint32_t t = __umulhi(rp.tc_mul, n);
+  return (int)((t + ((n - t) >> 1)) >> (rp.tc_sh - 1));
+}
 
 }  // namespace zh

@@ -26,7 +26,7 @@ struct TileGeom {
 template <bool kRep = true>
 __device__ __forceinline__ TileGeom tile_geom(const RasterP& rp, const Geo& g, int tile) {
   TileGeom t;
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int trl = tile_row(rp, tile), tc = tile - trl * rp.TC;
   t.r0 = (int64_t)(rp.tr0 + trl) * rp.T;
   t.h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - t.r0);
   t.c0 = (int64_t)tc * rp.T;

@@ -115,7 +115,7 @@ __device__ __forceinline__ void pip_cells_body(const PipP& p, int64_t pair_idx, 
   const RasterP& rp = p.rp;
   const int2 pr = p.isect[pair_idx];
   const int tile = pr.x, k = pr.y;
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int trl = tile_row(rp, tile), tc = tile - trl * rp.TC;
   const int64_t r0 = (int64_t)(rp.tr0 + trl) * rp.T, c0 = (int64_t)tc * rp.T;
   const int h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - r0);
   const int w = (int)min((int64_t)rp.T, rp.cols - c0);
@@ -268,7 +268,7 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
   const int2 pr0 = p.isect[pi0];
   const int tile = pr0.x;
   const int kp0 = pr0.y, kp1 = m > 1 ? p.isect[pi0 + 1].y : -1;
-  const int trl = tile / rp.TC, tc = tile - trl * rp.TC;
+  const int trl = tile_row(rp, tile), tc = tile - trl * rp.TC;
   const int64_t r0 = (int64_t)(rp.tr0 + trl) * rp.T, c0 = (int64_t)tc * rp.T;
   const int h = (int)min((int64_t)rp.T, rp.row0 + rp.nrows - r0);
   const int w = (int)min((int64_t)rp.T, rp.cols - c0);
