@@ -31,6 +31,9 @@
 #ifndef ZH_MIX_PF
 #define ZH_MIX_PF 0  // k_mixed_cells: L2 prefetch distance in main-loop iterations (0 = none)
 #endif
+#ifndef ZH_MIX_WIDE
+#define ZH_MIX_WIDE 1  // k_mixed_cells: 16-cell segments with 32-byte loads (flat layout)
+#endif
 #ifndef ZH_MIX_NOZERO
 #define ZH_MIX_NOZERO 0
 #endif
@@ -60,6 +63,7 @@ struct PipP {
   const int2* grp;       // tile groups of the cell kernel: {first pair index, #pairs (1 or 2)}
   int offb;              // k_mixed_cells: word offset of the second histogram (B)
   int bmo;               // k_mixed_cells: word offset of the two staged bitmaps
+  int wide;              // k_mixed_cells: 32-byte loads apply (raster base and pitch 32-byte aligned)
 };
 
 struct Ctx;  // zh_ctx.h
@@ -341,6 +345,60 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
     }
     const bool overlap = __syncthreads_or(ov != 0) != 0;
     const int16_t* base = rp.data + (r0 + cr - rp.row0) * pitch + k0 * 8;
+#if ZH_MIX_WIDE
+    // Flat layout, no overlap, 32-byte aligned rows: each thread takes 16-cell segments (one 32-byte
+    // load, one bitmap word for both halves), two rows in flight (the same 64 bytes and registers as
+    // four 16-byte vectors, half the load and bitmap instructions).
+    if constexpr (kCode == 2 && kMode >= 2) {
+      if (p.wide && !overlap && (c0 & 15) == 0) {
+        const int nk2 = (w + 15) >> 4;
+        if (nk2 <= (int)blockDim.x) {
+          const int rpi2 = blockDim.x / nk2;
+          const int kk2 = threadIdx.x % nk2, rs2 = threadIdx.x / nk2;
+          if (rs2 < rpi2) {
+            const int lc0 = kk2 * 16;  // multiple of 16: within one bitmap word
+            const int wi = lc0 >> 5, bsh = lc0 & 31;
+            uint32_t cskip16 = 0;
+            if (lc0 + 16 > w) cskip16 = (0xFFFFu << max(0, w - lc0)) & 0xFFFFu;
+            const int16_t* ptr = rp.data + (r0 + cr - rp.row0 + rs2) * pitch + c0 + lc0;
+            const int64_t step = (int64_t)rpi2 * pitch;
+            const uint2* bw = reinterpret_cast<const uint2*>(bm0) + rs2 * wpo + wi;
+            const int bstride = rpi2 * wpo;
+            int lr = rs2;
+            auto bits16 = [&](int u, uint32_t& s16, uint32_t& b16) {
+              const uint2 v = bw[u * bstride];
+              const uint32_t a = (v.x >> bsh) & 0xFFFFu;
+              b16 = (v.y >> bsh) & 0xFFFFu;
+              s16 = cskip16 | (~(a | b16) & 0xFFFFu);
+            };
+            for (; lr + rpi2 < ch; lr += 2 * rpi2, ptr += 2 * step, bw += 2 * bstride) {
+              uint32_t s0, e0, s1, e1;
+              bits16(0, s0, e0);
+              bits16(1, s1, e1);
+              uint4 q0l = make_uint4(0, 0, 0, 0), q0h = q0l, q1l = q0l, q1h = q0l;
+              if (s0 != 0xFFFFu) ld_stream32(ptr, q0l, q0h);
+              if (s1 != 0xFFFFu) ld_stream32(ptr + step, q1l, q1h);
+              if ((s0 & 0xFFu) != 0xFFu) count_sel(q0l, s0 & 0xFFu, e0 & 0xFFu);
+              if ((s0 >> 8) != 0xFFu) count_sel(q0h, s0 >> 8, e0 >> 8);
+              if ((s1 & 0xFFu) != 0xFFu) count_sel(q1l, s1 & 0xFFu, e1 & 0xFFu);
+              if ((s1 >> 8) != 0xFFu) count_sel(q1h, s1 >> 8, e1 >> 8);
+            }
+            for (; lr < ch; lr += rpi2, ptr += step, bw += bstride) {
+              uint32_t s0, e0;
+              bits16(0, s0, e0);
+              if (s0 == 0xFFFFu) continue;
+              uint4 ql, qh;
+              ld_stream32(ptr, ql, qh);
+              if ((s0 & 0xFFu) != 0xFFu) count_sel(ql, s0 & 0xFFu, e0 & 0xFFu);
+              if ((s0 >> 8) != 0xFFu) count_sel(qh, s0 >> 8, e0 >> 8);
+            }
+          }
+          __syncthreads();
+          continue;
+        }
+      }
+    }
+#endif
     const int hrem = h - cr;  // rows of the tile from this chunk on (prefetch bound)
     (void)hrem;
     if (nk <= (int)blockDim.x) {
