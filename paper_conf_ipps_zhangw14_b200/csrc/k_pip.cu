@@ -114,7 +114,6 @@ PipP pip_params(Ctx& c, const int2* pairs, const int64_t* n_dev) {
   p.grp = nullptr;
   p.offb = 0;
   p.bmo = 0;
-  p.wide = ((uintptr_t)c.rp.data % 32 == 0 && c.rp.pitch % 16 == 0) ? 1 : 0;
   return p;
 }
 

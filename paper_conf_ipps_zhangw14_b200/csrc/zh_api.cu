@@ -339,6 +339,7 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   c->rp.tr0 = (int32_t)tr0;
   c->rp.TRn = (int32_t)TRn;
   zh::set_tc_div(c->rp);
+  c->rp.wide = ((uintptr_t)c->rp.data % 32 == 0 && c->rp.pitch % 16 == 0) ? 1 : 0;
   c->geo = zh::Geo{r->gt[0], r->gt[1], r->gt[3], r->gt[5], o->rep_custom ? o->rep_x : 0.5,
                    o->rep_custom ? o->rep_y : 0.5, 1.0 / r->gt[1], 1.0 / r->gt[5]};
   c->on_host = r->on_host != 0;

@@ -372,6 +372,7 @@ struct RasterP {
   int64_t rows, cols, pitch, row0, nrows;
   int32_t T, TC, tr0, TRn;  // tile size, tile columns, first tile row, tile rows in shard
   uint32_t tc_mul, tc_sh;   // tile / TC by multiply-high (set_tc_div; Granlund-Montgomery round-up)
+  int32_t wide;             // 32-byte loads apply: data and pitch keep every 16-cell segment 32-byte aligned
 };
 
 // tc_mul / tc_sh for an exact n / TC, n < 2^31, with one multiply-high instead of a division loop.

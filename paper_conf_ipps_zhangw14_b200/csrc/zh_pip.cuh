@@ -63,7 +63,6 @@ struct PipP {
   const int2* grp;       // tile groups of the cell kernel: {first pair index, #pairs (1 or 2)}
   int offb;              // k_mixed_cells: word offset of the second histogram (B)
   int bmo;               // k_mixed_cells: word offset of the two staged bitmaps
-  int wide;              // k_mixed_cells: 32-byte loads apply (raster base and pitch 32-byte aligned)
 };
 
 struct Ctx;  // zh_ctx.h
@@ -350,7 +349,7 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
     // load, one bitmap word for both halves), two rows in flight (the same 64 bytes and registers as
     // four 16-byte vectors, half the load and bitmap instructions).
     if constexpr (kCode == 2 && kMode >= 2) {
-      if (p.wide && !overlap && (c0 & 15) == 0) {
+      if (rp.wide && !overlap && (c0 & 15) == 0) {
         const int nk2 = (w + 15) >> 4;
         if (nk2 <= (int)blockDim.x) {
           const int rpi2 = blockDim.x / nk2;

@@ -2,6 +2,10 @@
 #pragma once
 #include "zh_internal.cuh"
 
+#ifndef ZH_TILE_WIDE
+#define ZH_TILE_WIDE 1
+#endif
+
 namespace zh {
 
 // Histogram of one tile (tile-row trl, tile-column tc of the shard) into the shared histogram
@@ -32,6 +36,35 @@ __device__ __forceinline__ void tile_histogram(uint32_t* __restrict__ sh, const 
   const int16_t* base = rp.data + (r0 - rp.row0) * rp.pitch + k0 * 8;
   const int64_t pitch = rp.pitch;
 
+#if ZH_TILE_WIDE
+  // 16-cell segments, one 32-byte load each (sm_100 LDG.256), two rows in flight: the same bytes
+  // and registers as four 16-byte vectors with half the load instructions (full, aligned tiles)
+  if (kMode >= 2 && rp.wide && (c0 & 15) == 0 && (w & 15) == 0 && (w >> 4) <= (int)blockDim.x) {
+    const int nk2 = w >> 4, rpi2 = blockDim.x / nk2;
+    const int kk2 = threadIdx.x % nk2, rs2 = threadIdx.x / nk2;
+    if (rs2 < rpi2) {
+      const int16_t* p = rp.data + (r0 - rp.row0 + rs2) * rp.pitch + c0 + kk2 * 16;
+      const int64_t step = (int64_t)rpi2 * rp.pitch;
+      int r = rs2;
+      for (; r + rpi2 < h; r += 2 * rpi2, p += 2 * step) {
+        uint4 a0, a1, b0, b1;
+        ld_stream32(p, a0, a1);
+        ld_stream32(p + step, b0, b1);
+        count8_fast<kMode - 2, false>(sh, a0, 0, fb, dum2);
+        count8_fast<kMode - 2, false>(sh, a1, 0, fb, dum2);
+        count8_fast<kMode - 2, false>(sh, b0, 0, fb, dum2);
+        count8_fast<kMode - 2, false>(sh, b1, 0, fb, dum2);
+      }
+      for (; r < h; r += rpi2, p += step) {
+        uint4 a0, a1;
+        ld_stream32(p, a0, a1);
+        count8_fast<kMode - 2, false>(sh, a0, 0, fb, dum2);
+        count8_fast<kMode - 2, false>(sh, a1, 0, fb, dum2);
+      }
+    }
+    return;
+  }
+#endif
   if (nk <= (int)blockDim.x) {
     const int rpi = blockDim.x / nk;  // rows per block iteration
     const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
