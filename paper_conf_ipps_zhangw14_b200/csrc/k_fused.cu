@@ -242,7 +242,7 @@ __global__ void __launch_bounds__(512, ZH_PURE_MINB) k_fused_pure(PureP f) {
   for (int j = 0; j < nrun; ++j) {
     const int tile = s_tile[j];
     const int trl = tile_row(f.rp, tile), tc = tile - trl * f.rp.TC;
-    tile_histogram<kMode>(sh, f.rp, f.bp, f.fb, trl, tc);
+    tile_histogram<kMode, ZH_PURE_WROWS>(sh, f.rp, f.bp, f.fb, trl, tc);
     if (s_flush[j]) {  // uniform over the CTA
       __syncthreads();
       pure_flush<kU64>(f, tile, sh);

@@ -34,6 +34,9 @@
 #ifndef ZH_MIX_WIDE
 #define ZH_MIX_WIDE 1  // k_mixed_cells: 16-cell segments with 32-byte loads (flat layout)
 #endif
+#ifndef ZH_MIX_WROWS
+#define ZH_MIX_WROWS 2  // rows (32-byte loads) in flight per thread in that path
+#endif
 #ifndef ZH_MIX_NOZERO
 #define ZH_MIX_NOZERO 0
 #endif
@@ -370,17 +373,22 @@ __device__ __forceinline__ void mixed_cells_body(const PipP& p, int64_t g, uint3
               b16 = (v.y >> bsh) & 0xFFFFu;
               s16 = cskip16 | (~(a | b16) & 0xFFFFu);
             };
-            for (; lr + rpi2 < ch; lr += 2 * rpi2, ptr += 2 * step, bw += 2 * bstride) {
-              uint32_t s0, e0, s1, e1;
-              bits16(0, s0, e0);
-              bits16(1, s1, e1);
-              uint4 q0l = make_uint4(0, 0, 0, 0), q0h = q0l, q1l = q0l, q1h = q0l;
-              if (s0 != 0xFFFFu) ld_stream32(ptr, q0l, q0h);
-              if (s1 != 0xFFFFu) ld_stream32(ptr + step, q1l, q1h);
-              if ((s0 & 0xFFu) != 0xFFu) count_sel(q0l, s0 & 0xFFu, e0 & 0xFFu);
-              if ((s0 >> 8) != 0xFFu) count_sel(q0h, s0 >> 8, e0 >> 8);
-              if ((s1 & 0xFFu) != 0xFFu) count_sel(q1l, s1 & 0xFFu, e1 & 0xFFu);
-              if ((s1 >> 8) != 0xFFu) count_sel(q1h, s1 >> 8, e1 >> 8);
+            constexpr int WR = ZH_MIX_WROWS;
+            for (; lr + (WR - 1) * rpi2 < ch; lr += WR * rpi2, ptr += WR * step, bw += WR * bstride) {
+              uint32_t sv[WR], ev[WR];
+              uint4 ql[WR], qh[WR];
+#pragma unroll
+              for (int u = 0; u < WR; ++u) {
+                bits16(u, sv[u], ev[u]);
+                ql[u] = make_uint4(0, 0, 0, 0);
+                qh[u] = ql[u];
+                if (sv[u] != 0xFFFFu) ld_stream32(ptr + u * step, ql[u], qh[u]);
+              }
+#pragma unroll
+              for (int u = 0; u < WR; ++u) {
+                if ((sv[u] & 0xFFu) != 0xFFu) count_sel(ql[u], sv[u] & 0xFFu, ev[u] & 0xFFu);
+                if ((sv[u] >> 8) != 0xFFu) count_sel(qh[u], sv[u] >> 8, ev[u] >> 8);
+              }
             }
             for (; lr < ch; lr += rpi2, ptr += step, bw += bstride) {
               uint32_t s0, e0;
