@@ -121,6 +121,23 @@ def measured_peaks() -> dict:
     return {"hbm_gbs": 6650.0, "source": "fallback (B200_PROFILING.md)"}
 
 
+def read_ceiling():
+    """Read-only ceiling of the tile access pattern (no histogram: 16-byte loads of 256 x 256 tiles,
+    runs of 8 tiles per CTA, XOR only) measured on a B200 by tools/microbench/tile_read_bw.cu and
+    committed as profiles/r02/microbench_tile_read_bw.txt; the copy peak of MEASURED_PEAKS.json counts
+    read + write bytes, which a kernel that only reads can exceed."""
+    p = os.path.join(ROOT, "profiles", "r02", "microbench_tile_read_bw.txt")
+    if not os.path.exists(p):
+        return None
+    best = None
+    for line in open(p):
+        if "run 8" in line and "GB/s" in line:
+            v = float(line.split("=")[-1].split()[0])
+            best = v if best is None else max(best, v)
+    return (best, "tools/microbench/tile_read_bw.cu, runs of 8 tiles (profiles/r02/microbench_tile_read_bw.txt)") \
+        if best else None
+
+
 def traffic_from_profile(kernel_key: str, config: str, tile: int, path: str):
     """dram read+write bytes per launch of the dominant kernel from the committed ncu --set full
     capture of THIS configuration (profiles/ncu_traffic.json: {"<config>/T<tile>/<path>": {kernel:
@@ -442,6 +459,9 @@ def main():
                 "traffic": traffic_from_profile(dom, cfg.name, T, path) if world == 1 else None,
                 "peak_source": peaks["source"], "alg_bytes_per_launch": dom_b,
                 "share_of_step": dom_ms / ms if ms > 0 else None}
+    rc = read_ceiling()
+    if rc is not None:  # the copy peak counts read + write bytes; these kernels only read
+        roofline["read_ceiling"] = {"value": rc[0], "unit": "GB/s", "frac": achieved / rc[0], "source": rc[1]}
     log(f"timed ({path}): {ms:.3f} ms/step, {steps_detail}")
 
     # the other path, timed the same way (every SURVEY §8a row measured); not the headline
