@@ -1,5 +1,9 @@
 // zh_api.cu — the C ABI of libzh (include/zh.h): validation, context lifetime, step orchestration.
 #include <float.h>
+
+#ifndef ZH_DEVICE_SCAN
+#define ZH_DEVICE_SCAN 1  // zh_create: the vertex scan of large inputs on the device
+#endif
 #include <math.h>
 #include <stdarg.h>
 #include <stdio.h>
@@ -233,6 +237,31 @@ static zh_status validate(const zh_raster* r, const zh_polygons* p, const zh_bin
 // split over host threads for large inputs (CONUS: 9.6 M vertices, ~25 ms on one core).  zh_create
 // runs it before any CUDA call for small inputs, and for large ones while the vertex arrays are
 // already on their way to the device (the DMA hides the scan).
+static zh_status scan_verdict(const zh_raster* r, double amax, int64_t bad);
+
+// Large inputs (ZH_DEVICE_SCAN): the same scan on the device right after the vertices' H2D (the host
+// pass competed with the copy for host memory bandwidth: CONUS H2D 35 -> ~55 GB/s); the result comes
+// back with zh_create's closing synchronisation.  out[0] = bits of max |coordinate| (non-negative
+// doubles order like their bit patterns), out[1] = first non-finite vertex (INT64_MAX: none).
+__global__ void k_scan_vertices(const double* __restrict__ x, const double* __restrict__ y, int64_t n,
+                                unsigned long long* __restrict__ out) {
+  double m = 0.0;
+  long long bad = 0x7FFFFFFFFFFFFFFFll;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const double ax = fabs(x[i]), ay = fabs(y[i]);
+    if (!(ax <= DBL_MAX) || !(ay <= DBL_MAX)) bad = min(bad, (long long)i);
+    else m = fmax(m, fmax(ax, ay));
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+    bad = min(bad, __shfl_xor_sync(0xffffffffu, bad, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMax(&out[0], (unsigned long long)__double_as_longlong(m));
+    atomicMin(reinterpret_cast<long long*>(&out[1]), bad);
+  }
+}
+
 static zh_status scan_vertices(const zh_raster* r, const zh_polygons* p) {
   const int64_t nv = p->n_vert;
   const int nth = nv >= (1 << 20) ? (int)std::min<unsigned>(16u, std::max(1u, std::thread::hardware_concurrency())) : 1;
@@ -259,10 +288,17 @@ static zh_status scan_vertices(const zh_raster* r, const zh_polygons* p) {
     for (auto& x : th) x.join();
   }
   double amax = 0.0;
+  int64_t bad = -1;
   for (int t = 0; t < nth; ++t) {
-    if (part_bad[t] >= 0) return fail(ZH_ERR_INVALID_ARG, "non-finite vertex %lld", (long long)part_bad[t]);
+    if (part_bad[t] >= 0 && bad < 0) bad = part_bad[t];
     amax = std::max(amax, part_max[t]);
   }
+  return scan_verdict(r, amax, bad);
+}
+
+// bad >= 0: the first non-finite vertex
+static zh_status scan_verdict(const zh_raster* r, double amax, int64_t bad) {
+  if (bad >= 0) return fail(ZH_ERR_INVALID_ARG, "non-finite vertex %lld", (long long)bad);
   amax = std::max(amax, std::max(fabs(r->gt[0]), fabs(r->gt[3])));
   amax = std::max(amax, std::max(fabs(r->gt[0] + (double)r->cols * r->gt[1]), fabs(r->gt[3] + (double)r->rows * r->gt[5])));
   // The classification proof and the quick left/right edge tests need the cell size to dwarf the
@@ -378,7 +414,19 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
         (e = cudaMemcpyAsync(c->d_y.p, p->y, (size_t)p->n_vert * 8, cudaMemcpyHostToDevice, c->stream)))
       return cleanup_fail(cuda_fail(e, "zh_create (vertices H2D)"));
   }
+#if ZH_DEVICE_SCAN
+  if (scan_during_h2d) {  // on the device behind the copies; checked after the closing sync
+    if ((e = c->d_scan.ensure(16)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (scan)"));
+    const unsigned long long init[2] = {0ull, 0x7FFFFFFFFFFFFFFFull};
+    if ((e = cudaMemcpyAsync(c->d_scan.p, init, sizeof(init), cudaMemcpyHostToDevice, c->stream)) != cudaSuccess)
+      return cleanup_fail(cuda_fail(e, "zh_create (scan)"));
+    k_scan_vertices<<<148 * 8, 256, 0, c->stream>>>(c->d_x.as<double>(), c->d_y.as<double>(), p->n_vert,
+                                                     c->d_scan.as<unsigned long long>());
+    c->launches += 1;
+  }
+#else
   if (scan_during_h2d && (st = scan_vertices(r, p)) != ZH_OK) return cleanup_fail(st);
+#endif
   // output (the per-tile histograms of step 1 are allocated by the first zh_tile_hist)
   const size_t out_bytes = (size_t)p->n_poly * b->nbins * (c->out_u64 ? 8 : 4);
   if ((e = c->d_out_own.ensure(out_bytes)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (output)"));
@@ -407,8 +455,22 @@ extern "C" zh_status zh_create(zh_ctx* out, const zh_raster* r, const zh_polygon
   // the polygon arrays are the caller's (zh.h: they may be freed or reused once zh_create
   // returns); with page-locked host arrays the copies above are truly asynchronous
   ZH_TRC("enqueue");
+#if ZH_DEVICE_SCAN
+  if (scan_during_h2d &&
+      (e = cudaMemcpyAsync(c->pinned_counts, c->d_scan.p, 16, cudaMemcpyDeviceToHost, c->stream)) != cudaSuccess)
+    return cleanup_fail(cuda_fail(e, "zh_create (scan)"));
+#endif
   if ((e = cudaStreamSynchronize(c->stream)) != cudaSuccess) return cleanup_fail(cuda_fail(e, "zh_create (H2D)"));
   ZH_TRC("sync");
+#if ZH_DEVICE_SCAN
+  if (scan_during_h2d) {
+    const uint64_t* sc = reinterpret_cast<const uint64_t*>(c->pinned_counts);
+    double amax;
+    memcpy(&amax, &sc[0], 8);
+    const int64_t bad = sc[1] == 0x7FFFFFFFFFFFFFFFull ? -1 : (int64_t)sc[1];
+    if ((st = scan_verdict(r, amax, bad)) != ZH_OK) return cleanup_fail(st);
+  }
+#endif
   *out = reinterpret_cast<zh_ctx>(c);
   return ZH_OK;
 }
@@ -429,7 +491,7 @@ extern "C" void zh_destroy(zh_ctx h) {
                       &c->d_cub, &c->d_tile_hist, &c->d_out_own, &c->d_mixed, &c->d_pure_cnt,
                       &c->d_pure_cur, &c->d_pure_pk, &c->d_pure_off, &c->d_pure_poly, &c->d_pure_tiles,
                       &c->d_extra, &c->d_extra_pos, &c->d_pip, &c->d_pip_cur, &c->d_pbits, &c->d_remap, &c->d_fcounts, &c->d_stats,
-                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_band_poly, &c->d_band_first, &c->d_flag, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
+                      &c->d_pip_grp, &c->d_mixed_pk, &c->d_band_poly, &c->d_band_first, &c->d_scan, &c->d_flag, &c->d_need, &c->d_summary, &c->d_cdf, &c->d_dist, &c->d_ids};
   for (auto* b : bufs) b->release();
   ZH_TR("release");
   for (int i = 0; i < 16; ++i)
@@ -458,7 +520,7 @@ size_t zh::device_bytes(const Ctx& c) {
                             &c.d_cub, &c.d_tile_hist, &c.d_out_own, &c.d_mixed, &c.d_pure_cnt,
                             &c.d_pure_cur, &c.d_pure_pk, &c.d_pure_off, &c.d_pure_poly, &c.d_pure_tiles,
                             &c.d_extra, &c.d_extra_pos, &c.d_pip, &c.d_pip_cur, &c.d_pbits, &c.d_remap, &c.d_fcounts, &c.d_stats,
-                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_band_poly, &c.d_band_first, &c.d_flag, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
+                            &c.d_pip_grp, &c.d_mixed_pk, &c.d_band_poly, &c.d_band_first, &c.d_scan, &c.d_flag, &c.d_need, &c.d_summary, &c.d_cdf, &c.d_dist, &c.d_ids};
   size_t s = 0;
   for (auto* b : bufs) s += b->bytes;
   return s;

@@ -65,6 +65,7 @@ struct Ctx {
   DBuf d_band_cnt, d_band_off, d_band_cur, d_band_edges, d_class, d_flags, d_flag_pos;
   DBuf d_inside, d_isect, d_counts, d_cub;
   DBuf d_band_poly;  // band -> polygon
+  DBuf d_scan;  // zh_create: device vertex scan (max |coordinate| bits, first non-finite vertex)
   DBuf d_band_first;  // band -> #edges straddling its first row (at the front of its list), -1: unsorted
   // fused path lists (k_fused.cu)
   DBuf d_mixed, d_pure_cnt, d_pure_cur, d_pure_pk, d_pure_off, d_pure_poly, d_pure_tiles, d_extra, d_extra_pos,

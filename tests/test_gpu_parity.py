@@ -554,3 +554,32 @@ def test_random_configurations_fuzz(cuda_device, seed):
         got = z.output_device().cpu().numpy()
     got = got.view(np.uint64) if out_u64 else got.view(np.uint32)
     assert (got.astype(np.uint64) == H).all(), seed
+
+
+def test_large_polygon_set_validated_on_device(cuda_device):
+    """>= 2^20 vertices: zh_create scans them on the device behind their H2D (ZH_DEVICE_SCAN) — a
+    NaN or infinite vertex is rejected with its index, coordinates too large for the cell size are
+    UNSUPPORTED, and a clean set of that size equals the oracle."""
+    zh = _zh()
+    n = (1 << 20) + 7
+    th = np.linspace(0.0, 2.0 * np.pi, n, endpoint=False)
+    x, y = 32.0 + 20.5 * np.cos(th), 32.0 + 20.5 * np.sin(th)
+    gt = (0.0, 1.0, 0.0, 64.0, 0.0, -1.0)
+    spec = DemSpec(seed=3)
+    t = device_raster(spec, 64, 64)
+    bins = oracle.make_bins(256, nodata=-32768)
+    P = from_rings([[(x, y)]])
+    G = gpu_hist(t, gt, P, 256, 16, 64, nodata=-32768)
+    R = fill_host(spec, 64, 0, 0, 64, 64)
+    assert (G == oracle.o1(R, gt, P, bins)).all()
+    for bad, code in ((np.nan, zh.ZH_ERR_INVALID_ARG), (np.inf, zh.ZH_ERR_INVALID_ARG)):
+        xb = x.copy()
+        xb[777777] = bad
+        with pytest.raises(zh.ZhError) as ei:
+            zh.ZonalHistogram(t, gt, from_rings([[(xb, y)]]), 256, tile=16, cols=64, nodata=-32768)
+        assert ei.value.status == code and "777777" in str(ei.value)
+    # cell size 1 against |coordinate| ~ 2^31: the rounding of the coordinates is no longer far
+    # below a cell (zh_create's 2^-30 condition)
+    with pytest.raises(zh.ZhError) as ei:
+        zh.ZonalHistogram(t, gt, from_rings([[(x + 2.0 ** 31, y)]]), 256, tile=16, cols=64, nodata=-32768)
+    assert ei.value.status == zh.ZH_ERR_UNSUPPORTED
