@@ -61,6 +61,9 @@ __device__ __forceinline__ void crossing_row(uint32_t* __restrict__ bm, int wpr,
 // Shared-memory queue of long edges (more than kLongRows straddled rows in the chunk): they are
 // processed afterwards by whole warps, one row per lane, so that no thread serialises hundreds of
 // rows while the others wait at the barrier.
+#ifndef ZH_PAR_ST32
+#define ZH_PAR_ST32 1  // k_parity: 32-byte streaming stores of the parity rows
+#endif
 #ifndef ZH_PAR_DYN
 #define ZH_PAR_DYN 1  // k_parity: band edges claimed dynamically (atomic counter) after the first
 #endif
@@ -163,6 +166,18 @@ __device__ __forceinline__ void suffix_xor_store(const uint32_t* __restrict__ bm
       return v;
     };
     for (int wi = wpr - 1; wi >= wpo; --wi) carry ^= __popc(row[wi]) & 1u;  // "all cells" flips: parity only
+#if ZH_PAR_ST32
+    if ((wpo & 7) == 0) {  // 8 words per 32-byte streaming store (sm_100)
+      for (int g = wpo - 8; g >= 0; g -= 8) {
+        uint32_t v[8];
+#pragma unroll
+        for (int k = 7; k >= 0; --k) v[k] = step(row[g + k]);
+        asm volatile("st.global.cs.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(orow + g), "r"(v[0]), "r"(v[1]),
+                     "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+                     : "memory");
+      }
+    } else
+#endif
     if ((wpo & 3) == 0) {
       for (int g = wpo - 4; g >= 0; g -= 4) {
         uint4 v;
