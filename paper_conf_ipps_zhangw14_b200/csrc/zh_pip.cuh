@@ -152,6 +152,44 @@ __device__ __forceinline__ void pip_cells_body(const PipP& p, int64_t pair_idx, 
     }
     __syncthreads();
     const int16_t* base = rp.data + (r0 + cr - rp.row0) * pitch + k0 * 8;
+#if ZH_MIX_WIDE
+    // 16-cell segments with one 32-byte load each (as in k_mixed_cells), two rows in flight
+    if (kMode >= 2 && rp.wide && (c0 & 15) == 0 && ((w + 15) >> 4) <= (int)blockDim.x) {
+      const int nk2 = (w + 15) >> 4;
+      const int rpi2 = blockDim.x / nk2;
+      const int kk2 = threadIdx.x % nk2, rs2 = threadIdx.x / nk2;
+      if (rs2 < rpi2) {
+        const int lc0 = kk2 * 16;
+        const int wi = lc0 >> 5, bsh = lc0 & 31;
+        uint32_t cskip16 = 0;
+        if (lc0 + 16 > w) cskip16 = (0xFFFFu << max(0, w - lc0)) & 0xFFFFu;
+        const int16_t* ptr = rp.data + (r0 + cr - rp.row0 + rs2) * pitch + c0 + lc0;
+        const int64_t step = (int64_t)rpi2 * pitch;
+        int lr = rs2;
+        for (; lr + rpi2 < ch; lr += 2 * rpi2, ptr += 2 * step) {
+          const uint32_t s0 = cskip16 | (~(bm[lr * wpo + wi] >> bsh) & 0xFFFFu);
+          const uint32_t s1 = cskip16 | (~(bm[(lr + rpi2) * wpo + wi] >> bsh) & 0xFFFFu);
+          uint4 a0 = make_uint4(0, 0, 0, 0), a1 = a0, b0 = a0, b1 = a0;
+          if (s0 != 0xFFFFu) ld_stream32(ptr, a0, a1);
+          if (s1 != 0xFFFFu) ld_stream32(ptr + step, b0, b1);
+          if ((s0 & 0xFFu) != 0xFFu) count(a0, s0 & 0xFFu);
+          if ((s0 >> 8) != 0xFFu) count(a1, s0 >> 8);
+          if ((s1 & 0xFFu) != 0xFFu) count(b0, s1 & 0xFFu);
+          if ((s1 >> 8) != 0xFFu) count(b1, s1 >> 8);
+        }
+        for (; lr < ch; lr += rpi2, ptr += step) {
+          const uint32_t s0 = cskip16 | (~(bm[lr * wpo + wi] >> bsh) & 0xFFFFu);
+          if (s0 == 0xFFFFu) continue;
+          uint4 a0, a1;
+          ld_stream32(ptr, a0, a1);
+          if ((s0 & 0xFFu) != 0xFFu) count(a0, s0 & 0xFFu);
+          if ((s0 >> 8) != 0xFFu) count(a1, s0 >> 8);
+        }
+      }
+      __syncthreads();
+      continue;
+    }
+#endif
     if (nk <= (int)blockDim.x) {
       const int rpi = blockDim.x / nk;
       const int kk = threadIdx.x % nk, rs = threadIdx.x / nk;
