@@ -36,7 +36,7 @@ __device__ __forceinline__ double row_centre(const Geo& g, int64_t r) {
 }
 
 // Canonical edge (ya <= yb), Fig. 5 predicate in lower-endpoint-first orientation (R8).
-struct Edge {
+struct __align__(32) Edge {
   double xa, ya, xb, yb;
 };
 
