@@ -98,10 +98,10 @@ __device__ __forceinline__ int4 mbb_reduce(int k, int nv, double xmn, double xmx
       double rlo = fmax(floor(ra) - 1.0, (double)rp.row0);
       double rhi = fmin(floor(rb) + 1.0, (double)(rp.row0 + rp.nrows - 1));
       if (clo <= chi && rlo <= rhi) {
-        m.x = (int)((int64_t)clo / rp.T);
-        m.y = (int)((int64_t)chi / rp.T);
-        m.z = (int)((int64_t)rlo / rp.T);
-        m.w = (int)((int64_t)rhi / rp.T);
+        m.x = cell_tile(rp, (int64_t)clo);
+        m.y = cell_tile(rp, (int64_t)chi);
+        m.z = cell_tile(rp, (int64_t)rlo);
+        m.w = cell_tile(rp, (int64_t)rhi);
         nc = (int64_t)(m.y - m.x + 1) * (m.w - m.z + 1);
         nb = m.w - m.z + 1;
       }
@@ -144,7 +144,7 @@ __global__ void __launch_bounds__(256) k_mbb_edges(const int32_t* __restrict__ p
       edges[v] = e;
       const int2 rr = straddle_rows(g, e.ya, e.yb, rA, rB);
       erows[v] = rr;
-      span += (rr.x < rr.y) ? ((rr.y - 1) / T - rr.x / T + 1) : 0;
+      span += (rr.x < rr.y) ? (cell_tile(rp, rr.y - 1) - cell_tile(rp, rr.x) + 1) : 0;
     }
   }
   const int4 m = mbb_reduce(k, rvo[pro[k + 1]] - rvo[pro[k]], xmn, xmx, ymn, ymx, g, rp, mbb, ncand, nband);
@@ -163,7 +163,8 @@ __global__ void __launch_bounds__(256) k_mbb_edges(const int32_t* __restrict__ p
 constexpr int kSmemBands = 2048;
 __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ pro, const int32_t* __restrict__ rvo,
                                                     const int2* __restrict__ erows, const int4* __restrict__ mbb,
-                                                    const int64_t* __restrict__ band_base, int T, int mode,
+                                                    const int64_t* __restrict__ band_base, int T, uint32_t tmul,
+                                                    uint32_t tsh, int mode,
                                                     int32_t* __restrict__ band_cnt, const int32_t* __restrict__ band_off,
                                                     int32_t* __restrict__ band_edges, int32_t* __restrict__ band_poly,
                                                     int32_t* __restrict__ band_first) {
@@ -190,7 +191,8 @@ __global__ void __launch_bounds__(256) k_poly_bands(const int32_t* __restrict__ 
   for (int v = vb + threadIdx.x; v < ve; v += blockDim.x) {
     const int2 rr = erows[v];
     if (rr.x >= rr.y) continue;
-    for (int tr = rr.x / T; tr <= (rr.y - 1) / T; ++tr) {
+    const int tr1 = magic_q((uint32_t)(rr.y - 1), tmul, tsh);
+    for (int tr = magic_q((uint32_t)rr.x, tmul, tsh); tr <= tr1; ++tr) {
       const int i = tr - m.z;
       const int64_t r = (int64_t)tr * T;  // the band's first row
       const bool first = rr.x <= r && r < rr.y;
@@ -253,8 +255,8 @@ __global__ void __launch_bounds__(256) k_mark(const int32_t* __restrict__ pro, c
     const double rlo = fmax(floor(ra) - 1.0, (double)m.z * rp.T);
     const double rhi = fmin(floor(rb) + 1.0, (double)(m.w + 1) * rp.T - 1.0);
     if (clo > chi || rlo > rhi) continue;
-    const int tc_lo = (int)((int64_t)clo / rp.T), tc_hi = (int)((int64_t)chi / rp.T);
-    const int tr_lo = (int)((int64_t)rlo / rp.T), tr_hi = (int)((int64_t)rhi / rp.T);
+    const int tc_lo = cell_tile(rp, (int64_t)clo), tc_hi = cell_tile(rp, (int64_t)chi);
+    const int tr_lo = cell_tile(rp, (int64_t)rlo), tr_hi = cell_tile(rp, (int64_t)rhi);
     for (int tr = tr_lo; tr <= tr_hi; ++tr)
       for (int tc = tc_lo; tc <= tc_hi; ++tc) cls[base + (int64_t)(tr - m.z) * wk + (tc - m.x)] = 2;
   }
@@ -467,7 +469,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
   cudaMemsetAsync(c.d_band_cnt.p, 0, sizeof(int32_t) * ((size_t)nb + 1), c.stream);
   if (V > 0 && nb > 0) {
     k_poly_bands<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
-                                          c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 0,
+                                          c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, c.rp.t_mul, c.rp.t_sh, 0,
                                           c.d_band_cnt.as<int32_t>(), nullptr, nullptr, c.d_band_poly.as<int32_t>(),
                                           c.d_band_first.as<int32_t>());
     c.launches += 1;
@@ -478,7 +480,7 @@ cudaError_t launch_pairs_phase2(Ctx& c) {
     cudaMemcpyAsync(c.d_band_cur.p, c.d_band_off.p, sizeof(int32_t) * (size_t)nb, cudaMemcpyDeviceToDevice, c.stream);
     if (V > 0) {
       k_poly_bands<<<P, s2_threads(c), 0, c.stream>>>(c.d_pro.as<int32_t>(), c.d_rvo.as<int32_t>(), c.d_erows.as<int2>(),
-                                            c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, 1,
+                                            c.d_mbb.as<int4>(), c.d_band_base.as<int64_t>(), c.rp.T, c.rp.t_mul, c.rp.t_sh, 1,
                                             c.d_band_cur.as<int32_t>(), c.d_band_off.as<int32_t>(),
                                             c.d_band_edges.as<int32_t>(), nullptr, c.d_band_first.as<int32_t>());
       c.launches += 1;

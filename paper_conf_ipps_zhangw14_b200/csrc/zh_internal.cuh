@@ -373,23 +373,30 @@ struct RasterP {
   int32_t T, TC, tr0, TRn;  // tile size, tile columns, first tile row, tile rows in shard
   uint32_t tc_mul, tc_sh;   // tile / TC by multiply-high (set_tc_div; Granlund-Montgomery round-up)
   int32_t wide;             // 32-byte loads apply: data and pitch keep every 16-cell segment 32-byte aligned
+  uint32_t t_mul, t_sh;     // cell / T likewise
 };
 
-// tc_mul / tc_sh for an exact n / TC, n < 2^31, with one multiply-high instead of a division loop.
-__host__ inline void set_tc_div(RasterP& rp) {
-  const uint32_t d = (uint32_t)rp.TC;
+// (mul, sh) for an exact n / d, 0 <= n < 2^31, with one multiply-high instead of a division loop
+// (Granlund-Montgomery round-up): t = umulhi(mul, n), q = (t + ((n - t) >> 1)) >> (sh - 1); sh = 0: d = 1.
+__host__ inline void magic_div(uint32_t d, uint32_t& mul, uint32_t& sh) {
   uint32_t l = 0;
   while ((1ull << l) < d) ++l;  // ceil(log2 d)
-  rp.tc_sh = l;
-  rp.tc_mul = l == 0 ? 0u : (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+  sh = l;
+  mul = l == 0 ? 0u : (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+}
+__host__ inline void set_tc_div(RasterP& rp) {
+  magic_div((uint32_t)rp.TC, rp.tc_mul, rp.tc_sh);
+  magic_div((uint32_t)rp.T, rp.t_mul, rp.t_sh);
+}
+__device__ __forceinline__ int magic_q(uint32_t n, uint32_t mul, uint32_t sh) {
+  if (sh == 0) return (int)n;
+  const uint32_t t = __umulhi(mul, n);
+  return (int)((t + ((n - t) >> 1)) >> (sh - 1));
 }
 
 // (tile row, tile column) of a shard-local tile index
-__device__ __forceinline__ int tile_row(const RasterP& rp, int tile) {
-  const uint32_t n = (uint32_t)tile;
-  if (rp.tc_sh == 0) return tile;
-  const uint32_t t = __umulhi(rp.tc_mul, n);
-  return (int)((t + ((n - t) >> 1)) >> (rp.tc_sh - 1));
-}
+__device__ __forceinline__ int tile_row(const RasterP& rp, int tile) { return magic_q((uint32_t)tile, rp.tc_mul, rp.tc_sh); }
+// tile row / column of a (non-negative) cell row / column
+__device__ __forceinline__ int cell_tile(const RasterP& rp, int64_t cell) { return magic_q((uint32_t)cell, rp.t_mul, rp.t_sh); }
 
 }  // namespace zh
